@@ -1,0 +1,193 @@
+"""Pins for the planner oracle (oracle/planner.py): Eqs. (2), (7), (8), Listings 3/5, model.
+
+Independent references: per-block brute force over every thread x tap (which checks a
+block really needs), the paper's Listings 3 and 5 transcribed verbatim into
+tests/golden/ and executed literally, and closed-form limits of the model.
+"""
+import os
+import re
+
+import pytest
+
+from oracle import planner as P
+
+GOLDEN = os.path.join(os.path.dirname(__file__), "golden")
+
+
+def _compile_listing(path):
+    """Turn the transcribed CUDA listing into a Python function region(bx, by, wid, env)."""
+    lines = [l.rstrip() for l in open(path) if l.strip() and not l.lstrip().startswith("#")]
+    py = ["def region(bx, by, wid, BH_L, BH_R, BH_T, BH_B, W_L, W_R):"]
+    # An `if (c)` without a same-line goto governs the following indented lines (Listing 5's
+    # layout) or, if the next line is not indented, that single next line (Listing 3's).
+    pending_single = False
+    for k, l in enumerate(lines):
+        ind = len(l) - len(l.lstrip())
+        s = l.strip()
+        s = s.replace("blockIdx.x", "bx").replace("blockIdx.y", "by").replace("warpID.x", "wid")
+        s = s.replace("&&", "and")
+        depth = 1 + (1 if ind > 0 else 0) + (1 if pending_single else 0)
+        pending_single = False
+        m = re.match(r"if \((.*)\)\s*(goto (\w+);)?$", s)
+        if m:
+            cond, tgt = m.group(1), m.group(3)
+            if tgt:
+                py.append("    " * depth + f"if {cond}: return '{tgt}'")
+            else:
+                py.append("    " * depth + f"if {cond}:")
+                nxt = lines[k + 1]
+                pending_single = (len(nxt) - len(nxt.lstrip())) <= ind
+            continue
+        m = re.match(r"goto (\w+);$", s)
+        assert m, s
+        py.append("    " * depth + f"return '{m.group(1)}'")
+    env = {}
+    exec("\n".join(py), env)
+    return env["region"]
+
+
+LISTING3 = _compile_listing(os.path.join(GOLDEN, "listing3.txt"))
+LISTING5 = _compile_listing(os.path.join(GOLDEN, "listing5.txt"))
+
+SHAPES = [(sx, sy, m, n, tx, ty)
+          for (sx, sy) in [(7, 5), (16, 16), (23, 19), (39, 11)]
+          for (m, n) in [(1, 1), (3, 3), (5, 3), (7, 9)]
+          for (tx, ty) in [(1, 1), (4, 2), (8, 4), (16, 1)]]
+
+
+@pytest.mark.parametrize("sx,sy,m,n,tx,ty", SHAPES)
+def test_bounds_exact_vs_bruteforce(sx, sy, m, n, tx, ty):
+    """Eq. (2) (reading A2) is conservative AND tight: a block needs the L check iff
+    bx < BH_L, R iff bx >= BH_R, T iff by < BH_T, B iff by >= BH_B."""
+    b = P.bounds(sx, sy, m, n, tx, ty)
+    for by in range(b["NY"]):
+        for bx in range(b["NX"]):
+            need = P.needed_sides_bruteforce(sx, sy, m, n, tx, ty, bx, by)
+            assert ("L" in need) == (bx < b["BH_L"])
+            assert ("R" in need) == (bx >= b["BH_R"])
+            assert ("T" in need) == (by < b["BH_T"])
+            assert ("B" in need) == (by >= b["BH_B"])
+            if not b["degenerate"]:
+                reg, _ = P.listing3(bx, by, b)
+                assert need <= P.REGION_SIDES[reg]
+                assert need == P.REGION_SIDES[reg]          # and no superfluous check
+
+
+def test_printed_eq2_misses_checks():
+    """The literal Eq. (2) puts block 0 in Body for m=5, tx=32 although it
+    needs the left check -- the reason for reading A2."""
+    sx = sy = 128
+    bp = P.bounds_printed(sx, sy, 5, 5, 32, 32)
+    assert bp["BH_L"] == 0
+    assert "L" in P.needed_sides_bruteforce(sx, sy, 5, 5, 32, 32, 0, 1)
+    assert P.bounds(sx, sy, 5, 5, 32, 32)["BH_L"] == 1
+
+
+def test_degenerate_flag():
+    # cfg1 with a 64-wide tile: one block needs both the L and R check (A3).
+    b = P.bounds(64, 64, 3, 3, 64, 8)
+    assert b["degenerate"] and b["BH_R"] < b["BH_L"]
+    assert not P.bounds(64, 64, 3, 3, 32, 8)["degenerate"]
+
+
+@pytest.mark.parametrize("sx,sy,m,n,tx,ty", [s for s in SHAPES if not P.bounds(*s)["degenerate"]])
+def test_listing3_matches_paper_text(sx, sy, m, n, tx, ty):
+    b = P.bounds(sx, sy, m, n, tx, ty)
+    for by in range(b["NY"]):
+        for bx in range(b["NX"]):
+            assert P.listing3(bx, by, b)[0] == LISTING3(bx, by, 0, b["BH_L"], b["BH_R"], b["BH_T"],
+                                                        b["BH_B"], 0, 0)
+
+
+@pytest.mark.parametrize("sx,sy,m,n,tx,ty", [s for s in SHAPES if not P.bounds(*s)["degenerate"]])
+def test_eq8_counts(sx, sy, m, n, tx, ty):
+    """Eq. (8a)/(8b) (reading A17) equal a Listing 3 enumeration; they sum to N_block (Eq. 7)."""
+    b = P.bounds(sx, sy, m, n, tx, ty)
+    nb = P.n_block(b)
+    assert nb == P.n_block_enumerated(b)
+    assert sum(nb.values()) == b["NX"] * b["NY"]
+    assert all(v >= 0 for v in nb.values())
+
+
+def test_n_switch_table():
+    """Compares evaluated by Listing 3 under C short-circuit rules (A18)."""
+    assert P.n_switch_table() == {"TL": 2, "TR": 3, "T": 3, "BL": 6, "BR": 8, "B": 8, "R": 8,
+                                  "L": 9, "Body": 8}
+
+
+@pytest.mark.parametrize("sx,wx,m", [(512, 32, 3), (100, 8, 5), (77, 4, 7), (64, 16, 9), (256, 128, 31)])
+def test_warp_bounds_vs_bruteforce(sx, wx, m):
+    """Warp-grained bounds (a3/A22): warp column g needs L iff g < W_L, R iff g >= W_R."""
+    wb = P.warp_bounds(sx, m, wx)
+    hx = m // 2
+    for g in range(-(-sx // wx)):
+        xs = range(g * wx, (g + 1) * wx)           # launched threads (A10)
+        need_l = any(x - hx < 0 for x in xs)
+        need_r = any(x + hx >= sx for x in xs)
+        assert need_l == (g < wb["W_L"])
+        assert need_r == (g >= wb["W_R"])
+
+
+@pytest.mark.parametrize("sx,sy,m,n,tx,ty,wx", [(512, 64, 3, 3, 128, 4, 32), (300, 40, 5, 5, 64, 8, 16),
+                                                (1000, 30, 7, 3, 256, 2, 64), (96, 96, 9, 9, 32, 8, 8)])
+def test_listing5_matches_paper_and_is_safe(sx, sy, m, n, tx, ty, wx):
+    """Listing 5 evaluated on global warp columns: the paper's text and the
+    oracle agree, and each warp's region covers every check its pixels really need."""
+    b = P.bounds(sx, sy, m, n, tx, ty)
+    assert not b["degenerate"]
+    wb = P.warp_bounds(sx, m, wx)
+    wpb = tx // wx
+    hx, hy = m // 2, n // 2
+    for by in range(b["NY"]):
+        for bx in range(b["NX"]):
+            for w in range(wpb):
+                g = bx * wpb + w
+                reg, _ = P.listing5(bx, by, g, b, wb)
+                # golden text uses `warpID.x > W_L` with W_L = last checked warp (A22)
+                assert reg == LISTING5(bx, by, g, b["BH_L"], b["BH_R"], b["BH_T"], b["BH_B"],
+                                       wb["W_L"] - 1, wb["W_R"])
+                need = set()
+                for y in range(by * ty, (by + 1) * ty):      # launched threads (A10)
+                    for x in range(g * wx, (g + 1) * wx):
+                        if x - hx < 0: need.add("L")
+                        if x + hx >= sx: need.add("R")
+                        if y - hy < 0: need.add("T")
+                        if y + hy >= sy: need.add("B")
+                assert need <= P.REGION_SIDES[reg], (bx, by, w, reg, need)
+
+
+def test_listing5_paper_example():
+    """block of 128 threads = 4 warps, 3x3 operator: only the leftmost warp needs the
+    left check and only the rightmost the right check (one pixel per thread, wx = 32)."""
+    sx, sy = 512, 64
+    b = P.bounds(sx, sy, 3, 3, 128, 1)
+    wb = P.warp_bounds(sx, 3, 32)
+    regs = [P.listing5(g // 4, 5, g, b, wb)[0] for g in range(16)]
+    assert regs[0] == "L" and regs[-1] == "R" and set(regs[1:-1]) == {"Body"}
+    assert [P.listing3(g // 4, 5, b)[0] for g in range(16)][:4] == ["L"] * 4
+
+
+def test_fig3_trend():
+    """Fig. 3 / P:L173: for a 5x5 operator, smaller images have a lower share of Body blocks,
+    and a larger block leaves fewer Body blocks at the same size."""
+    for tile in [(32, 4), (128, 1), (128, 16)]:
+        fr = [P.body_fraction(s, s, 5, 5, *tile) for s in (512, 1024, 2048, 4096)]
+        assert fr == sorted(fr) and fr[0] < fr[-1] < 1.0
+    assert P.body_fraction(512, 512, 5, 5, 256, 16) < P.body_fraction(512, 512, 5, 5, 32, 4)
+
+
+def test_model_limits():
+    """Eq. (9)/(10) limits: with a 1-pixel image border share -> 0, form T gives
+    R -> (4c+k) m n / (ipc * n_sw(Body) + k m n) (threads = tx ty), approached monotonically;
+    G scales with O_ISP / O_naive."""
+    c, k, ipc = 4.0, 20.0, 2.0
+    m = n = 13
+    limit = (4 * c + k) * m * n / (ipc * 8 + k * m * n)
+    rs = [P.model(s, s, m, n, 32, 4, c, k, ipc_switch=ipc)["R_reduced"] for s in (512, 1024, 2048, 4096, 16384)]
+    assert rs == sorted(rs) and abs(rs[-1] - limit) / limit < 0.01 and rs[-1] < limit
+    g = P.model(2048, 2048, m, n, 32, 4, c, k, o_naive=1.0, o_isp=0.5, ipc_switch=ipc)
+    assert abs(g["G"] - 0.5 * g["R_reduced"]) < 1e-12
+    # form P (switch charged per tap) predicts R ~ 1 for this calibration (reading A14)
+    rp = P.model(4096, 4096, m, n, 32, 4, c, k, ipc_switch=ipc, form="P")["R_reduced"]
+    assert abs(rp - (4 * c + k) / (ipc * 8 + k)) / rp < 0.02
+    assert P.model(64, 64, 3, 3, 64, 8, c, k)["choice"] == "naive"      # degenerate
