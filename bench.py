@@ -1,0 +1,423 @@
+#!/usr/bin/env python
+"""Benchmark of the ISP hot path (BASELINE.json configs[1]) on B200.
+
+Step = one pass of the hot path over one batch: the 5x5 binomial Gaussian (f32) over a
+4096 x 4096 image in all four border modes (Clamp, Mirror, Repeat, Constant), variant
+AUTO ("isp+m": the Eq. (10) model picks ISP or naive), i.e. 4 kernel launches.
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl {isp,reference}]
+
+N = 1: the 4096^2 image.  N > 1 (torchrun, one rank per GPU, NCCL): weak scaling --
+each rank owns a 4096-row strip of a (4096 N) x 4096 image and exchanges 2-row halos
+with its neighbours (ring for Repeat) through isp_shard_filter_f32.
+value = output pixels of all ranks / max-over-ranks time (Mpixel/s).
+
+Timing: W untimed warm-up steps, then exactly K steps replayed from CUDA graphs
+(one graph per rotation phase), bracketed by barrier + synchronize, timed with CUDA
+events on the launch stream; inputs rotate over 6 in/out buffer pairs (768 MiB > 2x
+L2), so every launch reads cold HBM.  nvidia-smi clocks are sampled during the timed
+region.  --impl reference times the CPU oracle (oracle/, test infrastructure) on the
+host cores over a bounded sample of the same workload.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+METRIC = "Mpixel/s & HBM GB/s fraction per filter/border mode; ISP speedup vs naive"
+UNIT = "Mpixel/s"
+MODES = ["clamp", "mirror", "repeat", "constant"]
+N_SIDE = 4096
+WINDOW = 5
+CONST = 0.5
+NPAIRS = 6
+BYTES_PER_PX = 8          # algorithmic: one f32 read + one f32 write per output pixel
+
+
+def env_rank():
+    return int(os.environ.get("RANK", 0)), int(os.environ.get("WORLD_SIZE", 1)), int(os.environ.get("LOCAL_RANK", 0))
+
+
+def gauss_mask():
+    import synth
+    b = synth.binomial_row(WINDOW).astype(np.float64)
+    return (np.outer(b, b) / b.sum() ** 2).astype(np.float32)
+
+
+def peaks():
+    try:
+        return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
+    except Exception:
+        return {}
+
+
+def ncu_traffic():
+    """Per-launch DRAM bytes of the dominant kernel from the committed ncu --set full summary."""
+    p = os.path.join(ROOT, "profiles", "ncu_summary.json")
+    try:
+        d = json.load(open(p))
+        return d.get("dominant_kernel", {}).get("dram_bytes_per_launch")
+    except Exception:
+        return None
+
+
+class ClockSampler:
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, device_index):
+        self.dev = device_index
+        self.proc = None
+        self.path = os.path.join("/tmp", f"isp_clocks_{os.getpid()}.csv")
+
+    def __enter__(self):
+        try:
+            self.f = open(self.path, "w")
+            self.proc = subprocess.Popen(["nvidia-smi", f"--query-gpu={self.Q}", "--format=csv,noheader,nounits",
+                                          "-lms", "50", "-i", str(self.dev)], stdout=self.f,
+                                         stderr=subprocess.DEVNULL)
+            time.sleep(0.3)
+        except Exception:
+            self.proc = None
+        return self
+
+    def __exit__(self, *a):
+        if self.proc is not None:
+            time.sleep(0.1)
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except Exception:
+                self.proc.kill()
+            self.f.close()
+
+    def summary(self, t0, t1):
+        if self.proc is None:
+            return None
+        rows = []
+        for line in open(self.path):
+            parts = [p.strip() for p in line.split(",")]
+            if len(parts) < 9:
+                continue
+            try:
+                rows.append((float(parts[1]), float(parts[2]), parts[5:9]))
+            except ValueError:
+                continue
+        if not rows:
+            return None
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[k] for (_, _, r) in rows for k in range(4) if r[k].lower().startswith("active")})
+        loaded = [c for (c, _, _) in rows]
+        return {"sm_mhz": statistics.median(loaded), "sm_max_mhz": max(m for (_, m, _) in rows),
+                "reasons": reasons, "samples": len(rows)}
+
+
+def cpu_oracle_rate(target_s=12.0, threads=None):
+    """Oracle (oracle/ C, double accumulation, per-read border map) on the host cores over a
+    bounded row sample of the same workload, all four modes.  Returns dict for cpu_baseline."""
+    import oracle
+    import synth
+    threads = threads or os.cpu_count() or 1
+    oracle.build_oracle()
+    img = synth.uniform_f32(N_SIDE, N_SIDE, synth.CONFIG_SEEDS["cfg2"])
+    mask = gauss_mask()
+    # calibrate on 4 rows per mode
+    t = time.perf_counter()
+    for m in MODES:
+        oracle.filter_f64(img, mask, m, CONST, rows=(0, 4 * threads), threads=threads)
+    dt = time.perf_counter() - t
+    rows = int(max(threads, min(N_SIDE, 4 * threads * target_s / max(dt, 1e-6))))
+    rows -= rows % threads
+    rows = max(rows, threads)
+    y0 = (N_SIDE - rows) // 2
+    t = time.perf_counter()
+    for m in MODES:
+        oracle.filter_f64(img, mask, m, CONST, rows=(y0, y0 + rows), threads=threads)
+    dt = time.perf_counter() - t
+    px = 4 * rows * N_SIDE
+    return {"value": px / dt / 1e6, "unit": UNIT, "cores": threads, "kind": "oracle",
+            "sample": f"rows [{y0},{y0 + rows}) of the 4096x4096 cfg2 image x 4 modes ({px} px, {dt:.1f} s)",
+            "seconds": dt}
+
+
+# ------------------------------------------------------------------------------------------
+def run_reference(args):
+    rank, world, _ = env_rank()
+    if rank != 0:
+        return
+    import oracle
+    import synth
+    threads = os.cpu_count() or 1
+    oracle.build_oracle()
+    img = synth.uniform_f32(N_SIDE, N_SIDE, synth.CONFIG_SEEDS["cfg2"])
+    mask = gauss_mask()
+    # each step = a bounded sample (rows_per_step rows x 4 modes), sized so the run ends in minutes
+    rows_per_step = max(threads, 8 * threads // 8)
+    times = []
+    for k in range(args.warmup + args.steps):
+        y0 = (k * rows_per_step) % (N_SIDE - rows_per_step)
+        t = time.perf_counter()
+        for m in MODES:
+            oracle.filter_f64(img, mask, m, CONST, rows=(y0, y0 + rows_per_step), threads=threads)
+        if k >= args.warmup:
+            times.append(time.perf_counter() - t)
+    tot = sum(times)
+    px = 4 * rows_per_step * N_SIDE * args.steps
+    val = px / tot / 1e6
+    line = {"impl": "reference", "metric": METRIC, "value": val, "unit": UNIT, "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * tot / args.steps,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": "cfg2: 5x5 binomial Gaussian f32 4096x4096, 4 border modes (oracle sample)",
+                       "sample_rows_per_step": rows_per_step},
+            "cpu_baseline": {"value": val, "unit": UNIT, "cores": threads, "kind": "oracle",
+                             "sample": f"{rows_per_step} rows x 4096 px x 4 modes per step"},
+            "e2e": {"value": val, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+# ------------------------------------------------------------------------------------------
+def run_isp(args):
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_ipps_qiaoth21_b200 as isp
+    import synth
+
+    rank, world, local = env_rank()
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    isp.lib()
+    mask = gauss_mask()
+    H_img = N_SIDE * world
+    halo = WINDOW // 2
+    # ---- inputs: the seeded cfg2 image (rank r: its strip of the tall image) ----
+    host_img = synth.uniform_f32(N_SIDE, N_SIDE, synth.CONFIG_SEEDS["cfg2"] + rank)
+    pairs = []
+    for _ in range(NPAIRS):
+        if world > 1:
+            strip = torch.empty((N_SIDE + 2 * halo, N_SIDE), dtype=torch.float32, device=dev)
+            strip[halo:halo + N_SIDE].copy_(torch.from_numpy(host_img))
+            inp = strip
+        else:
+            inp = torch.from_numpy(host_img).to(dev)
+        out = torch.empty((N_SIDE, N_SIDE), dtype=torch.float32, device=dev)
+        pairs.append((inp, out))
+    ctx = None
+    comm_stream = torch.cuda.Stream(device=dev)
+    if world > 1:
+        uid = [isp.isp_shard_unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(uid, src=0)
+        ctx = isp.isp_shard_init(uid[0], rank, world, local)
+    stream = torch.cuda.Stream(device=dev)
+    variant = args.variant
+
+    def launch(mode, pair, v=variant):
+        inp, out = pairs[pair]
+        if world > 1:
+            isp.isp_shard_filter_f32(ctx, inp, H_img, halo, mask, mode, CONST, out=out, variant=v, stream=stream,
+                                     comm_stream=comm_stream)
+        else:
+            isp.isp_filter_ex(inp, mask, mode, CONST, out=out, variant=v, stream=stream)
+
+    def step(k, v=variant):
+        for i, m in enumerate(MODES):
+            launch(m, (4 * k + i) % NPAIRS, v)
+
+    launches_per_step = 4 * (len([l for l in isp.isp_shard_schedule(H_img, rank, world, halo, halo, 0)["launch"]
+                                  if l[1] > 0]) if world > 1 else 1)
+    nphase = NPAIRS // np.gcd(4, NPAIRS)          # rotation period in steps
+    use_graph = not args.no_graph
+
+    with torch.cuda.stream(stream):
+        for k in range(max(args.warmup, 1)):      # warm-up (also loads every kernel)
+            step(k)
+    torch.cuda.synchronize()
+    graphs = []
+    if use_graph:
+        try:
+            for ph in range(nphase):
+                g = torch.cuda.CUDAGraph()
+                with torch.cuda.graph(g, stream=stream):
+                    step(ph)
+                graphs.append(g)
+            for g in graphs:
+                g.replay()
+            torch.cuda.synchronize()
+        except Exception as e:  # pragma: no cover
+            print(f"[bench] graph capture failed ({e}); eager launches", file=sys.stderr)
+            graphs = []
+            use_graph = False
+
+    def run_steps(K, v=variant):
+        with torch.cuda.stream(stream):
+            for k in range(K):
+                if use_graph and v == variant:
+                    graphs[k % nphase].replay()
+                else:
+                    step(k, v)
+
+    plan = isp.isp_last_plan()
+    # ---- timed region ----
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    with ClockSampler(local) as cs:
+        t_wall0 = time.time()
+        e0.record(stream)
+        run_steps(args.steps)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        t_wall1 = time.time()
+    if world > 1:
+        dist.barrier()
+    ms = e0.elapsed_time(e1)
+    if world > 1:
+        t = torch.tensor([ms], device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms = float(t.item())
+    clocks = cs.summary(t_wall0, t_wall1)
+    px_step = 4 * N_SIDE * N_SIDE * world
+    value = px_step * args.steps / (ms / 1e3) / 1e6
+    ms_step = ms / args.steps
+
+    # ---- per-launch duration of the dominant kernel (the ISP 5x5 f32 stencil) ----
+    per_launch_us = 1e3 * ms_step / 4.0
+    pk = peaks()
+    hbm = pk.get("hbm_gbs")
+    achieved = BYTES_PER_PX * N_SIDE * N_SIDE / (per_launch_us * 1e-6) / 1e9
+    roof = {"bound": "hbm", "achieved": achieved, "peak": hbm if hbm else 6650.0, "unit": "GB/s",
+            "frac": achieved / (hbm if hbm else 6650.0), "traffic": ncu_traffic(),
+            "peak_source": "MEASURED_PEAKS.json hbm_gbs" if hbm else "fallback (B200_PROFILING.md)",
+            "kernel": "k_stencil<OpSepF32<5,5>> (ISP, separable 5x5 f32)",
+            "algorithmic_bytes_per_launch": BYTES_PER_PX * N_SIDE * N_SIDE,
+            "duration_us": per_launch_us,
+            "duration_method": "timed region / launches (graph replay, kernels back-to-back)"}
+
+    # ---- ISP vs naive per mode (same methodology, single-GPU variants) ----
+    variants = {}
+    if world == 1 and not args.quick:
+        for m in MODES:
+            variants[m] = {}
+            for v in ["auto", "warp", "block", "naive"]:
+                R = 12
+                g = torch.cuda.CUDAGraph()
+                with torch.cuda.stream(stream):
+                    for i in range(2):
+                        launch(m, i % NPAIRS, v)
+                torch.cuda.synchronize()
+                with torch.cuda.graph(g, stream=stream):
+                    for i in range(R):
+                        launch(m, i % NPAIRS, v)
+                torch.cuda.synchronize()
+                reps = 40
+                a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                with torch.cuda.stream(stream):
+                    g.replay()
+                    a.record(stream)
+                    for _ in range(reps):
+                        g.replay()
+                    b.record(stream)
+                torch.cuda.synchronize()
+                us = 1e3 * a.elapsed_time(b) / (reps * R)
+                variants[m][v] = {"us": us, "gbs": BYTES_PER_PX * N_SIDE * N_SIDE / (us * 1e-6) / 1e9,
+                                  "mpix_s": N_SIDE * N_SIDE / us}
+            variants[m]["speedup_isp_vs_naive"] = variants[m]["naive"]["us"] / variants[m]["warp"]["us"]
+            variants[m]["speedup_auto_vs_naive"] = variants[m]["naive"]["us"] / variants[m]["auto"]["us"]
+
+    # ---- end to end: pinned host buffers, H2D + filter + D2H inside the timed region ----
+    e2e = None
+    if not args.quick:
+        hin = torch.from_numpy(host_img).pin_memory()
+        houts = [torch.empty((N_SIDE, N_SIDE), dtype=torch.float32).pin_memory() for _ in range(2)]
+        E = max(3, min(20, args.steps // 100))
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        with torch.cuda.stream(stream):
+            a.record(stream)
+            for k in range(E):
+                for i, m in enumerate(MODES):
+                    inp, out = pairs[i % NPAIRS]
+                    dst = inp[halo:halo + N_SIDE] if world > 1 else inp
+                    dst.copy_(hin, non_blocking=True)
+                    if world > 1:
+                        isp.isp_shard_filter_f32(ctx, inp, H_img, halo, mask, m, CONST, out=out, stream=stream,
+                                                 comm_stream=comm_stream)
+                    else:
+                        isp.isp_filter(inp, mask, m, CONST, out=out, stream=stream)
+                    houts[i % 2].copy_(out, non_blocking=True)
+            b.record(stream)
+        torch.cuda.synchronize()
+        ems = a.elapsed_time(b)
+        if world > 1:
+            t = torch.tensor([ems], device=dev)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            ems = float(t.item())
+        e2e = {"value": px_step * E / (ems / 1e3) / 1e6, "unit": UNIT,
+               "h2d_bytes_per_step": 4 * N_SIDE * N_SIDE * 4, "d2h_bytes_per_step": 4 * N_SIDE * N_SIDE * 4,
+               "steps": E, "ms_per_step": ems / E, "api": "isp_filter via the Python binding, pinned host buffers"}
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu:
+        cpu = cpu_oracle_rate()
+
+    if ctx is not None:
+        torch.cuda.synchronize()
+        isp.isp_shard_destroy(ctx)
+    if rank == 0:
+        line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+                "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True, "scaling": "weak",
+                "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+                "config": {"workload": "cfg2: 5x5 binomial Gaussian f32 4096x4096 per rank, 4 border modes "
+                                       "(clamp, mirror, repeat, constant), variant auto (isp+m)"
+                                       + (f"; {world} ranks = row strips of a {H_img}x4096 image, NCCL halo exchange"
+                                          if world > 1 else ""),
+                           "image": [H_img, N_SIDE], "window": [WINDOW, WINDOW], "const": CONST,
+                           "l2": f"rotating {NPAIRS} in/out buffer pairs ({NPAIRS * 128} MiB > 2x L2)",
+                           "parallelism": f"row-strips x{world}" if world > 1 else "single GPU",
+                           "cuda_graphs": use_graph, "plan": {k: plan[k] for k in
+                                                              ("tile_w", "tile_h", "choice", "g", "degenerate")}},
+                "roofline": roof, "cpu_baseline": cpu, "e2e": e2e,
+                "gpu_launches": args.steps * launches_per_step, "clocks": clocks,
+                "isp_vs_naive": variants or None}
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=6000)
+    ap.add_argument("--warmup", type=int, default=20)
+    ap.add_argument("--impl", default="isp", choices=["isp", "reference"])
+    ap.add_argument("--variant", default="auto", choices=["auto", "warp", "block", "naive"])
+    ap.add_argument("--no-graph", action="store_true")
+    ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--quick", action="store_true", help="skip the variant table and e2e (profiling runs)")
+    args = ap.parse_args()
+    if args.warmup < 3:
+        ap.error("--warmup must be >= 3")
+    if args.impl == "reference":
+        run_reference(args)
+    else:
+        run_isp(args)
+
+
+if __name__ == "__main__":
+    main()

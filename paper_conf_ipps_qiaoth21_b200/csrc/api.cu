@@ -1,0 +1,696 @@
+// api.cu -- the C ABI (include/isp.h): validation, the region planner and analytic
+// model (Eqs. 2-10), variant selection ("isp+m") and kernel launch.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <mutex>
+#include <unordered_map>
+#include <vector>
+
+#include "../../include/isp.h"
+#include "internal.h"
+#include "kernels.h"
+
+using namespace ispk;
+
+namespace {
+
+thread_local char g_err[512] = "";
+thread_local isp_plan_info g_last_plan{};
+int g_override_wx = 0, g_override_ty = 0;
+
+}  // namespace
+
+isp_status_t ispi_fail(isp_status_t s, const char *fmt, ...)
+{
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(g_err, sizeof(g_err), fmt, ap);
+    va_end(ap);
+    return s;
+}
+
+namespace {
+#define fail ispi_fail
+
+isp_status_t cuda_status(cudaError_t e, const char *what)
+{
+    if (e == cudaSuccess) return ISP_OK;
+    if (e == cudaErrorNotSupported) return fail(ISP_EUNSUPPORTED, "%s: not built for this window", what);
+    return fail(ISP_ECUDA, "%s: %s", what, cudaGetErrorString(e));
+}
+
+long long floor_div(long long a, long long b) { return a >= 0 ? a / b : -((-a + b - 1) / b); }
+long long ceil_div(long long a, long long b) { return -floor_div(-a, b); }
+
+bool ranges_overlap(const void *a, size_t abytes, const void *b, size_t bbytes)
+{
+    const char *pa = (const char *)a, *pb = (const char *)b;
+    return pa < pb + bbytes && pb < pa + abytes;
+}
+
+size_t img_bytes(int w, int h, int pitch, size_t es) { return ((size_t)(h - 1) * pitch + w) * es; }
+
+isp_status_t check_geom(int w, int h, int pitch, int out_pitch, int mw, int mh, int mode)
+{
+    if (w < 1 || h < 1) return fail(ISP_EINVAL, "image size %dx%d", w, h);
+    if (pitch < w || out_pitch < w) return fail(ISP_EINVAL, "pitch %d / out_pitch %d < width %d", pitch, out_pitch, w);
+    if (mw < 1 || mh < 1 || mw > 31 || mh > 31 || (mw % 2) == 0 || (mh % 2) == 0)
+        return fail(ISP_EINVAL, "window %dx%d must be odd and in [1,31] (reading A8)", mw, mh);
+    if (mode < 0 || mode > 3) return fail(ISP_EINVAL, "border mode %d", mode);
+    return ISP_OK;
+}
+
+// ---------------------------------------------------------------------------------
+// Planner: Eq. (2) (reading A2), Eq. (7), Listing 5 warp bounds (A22), Eq. (8) (A17).
+// ---------------------------------------------------------------------------------
+struct Plan {
+    int px, wx, ty, tile_w, warp_w;
+    int nx, ny;
+    int bh_l, bh_r, bh_t, bh_b, w_l, w_r;
+    bool degenerate;
+};
+
+Plan make_plan(int w, int h, int hx, int hy, int px, int tile_w_req, int tile_h_req, int warp_w_req,
+               const RowRange *rr = nullptr)
+{
+    const RowRange whole{0, h, h, 1, 1};
+    if (!rr) rr = &whole;
+    Plan p{};
+    p.px = px;
+    const int warp_w = warp_w_req > 0 ? warp_w_req : 32 * px;
+    int wx;
+    if (tile_w_req > 0) {
+        wx = std::max(1, tile_w_req / warp_w);
+    } else if (g_override_wx > 0) {
+        wx = g_override_wx;
+    } else {
+        wx = (int)std::min<long long>(4, std::max<long long>(1, ceil_div(w, warp_w)));
+    }
+    int ty;
+    if (tile_h_req > 0) ty = tile_h_req;
+    else if (g_override_ty > 0) ty = g_override_ty;
+    else {
+        // enough tiles for >= ~4 waves of 148 SMs x 8 resident blocks, rows >= 8
+        const long long nxl = ceil_div(w, (long long)wx * warp_w);
+        ty = 32;
+        while (ty > 8 && nxl * ceil_div(rr->nrows, ty) < 148LL * 8) ty /= 2;
+    }
+    p.wx = wx;
+    p.ty = ty;
+    p.warp_w = warp_w;
+    p.tile_w = wx * warp_w;
+    p.nx = (int)ceil_div(w, p.tile_w);
+    p.ny = (int)ceil_div(rr->nrows, ty);
+    p.bh_l = (int)ceil_div(hx, p.tile_w);
+    p.bh_r = (int)floor_div(w - hx, p.tile_w);
+    // Eq. (2) in y, relative to the launch's first row oy0; only real image edges count.
+    p.bh_t = rr->t_real ? (int)std::max<long long>(0, ceil_div(hy - rr->oy0, ty)) : 0;
+    const long long safe_end = rr->b_real ? std::min<long long>(rr->oy0 + rr->nrows, (long long)h - hy)
+                                          : rr->oy0 + rr->nrows;
+    p.bh_b = (int)floor_div(safe_end - rr->oy0, ty);
+    p.w_l = (int)ceil_div(hx, warp_w);
+    p.w_r = (int)floor_div(w - hx, warp_w);
+    p.degenerate = p.bh_l > p.bh_r || p.bh_t > p.bh_b;
+    return p;
+}
+
+void n_block(const Plan &p, long long nb[9])
+{
+    const long long L = p.bh_l, R = p.bh_r, T = p.bh_t, B = p.bh_b, NX = p.nx, NY = p.ny;
+    nb[0] = L * T;                 // TL
+    nb[1] = (NX - R) * T;          // TR
+    nb[2] = (R - L) * T;           // T
+    nb[3] = L * (NY - B);          // BL
+    nb[4] = (NX - R) * (NY - B);   // BR
+    nb[5] = (R - L) * (NY - B);    // B
+    nb[6] = (NX - R) * (B - T);    // R
+    nb[7] = L * (B - T);           // L
+    long long s = 0;
+    for (int k = 0; k < 8; ++k) s += nb[k];
+    nb[8] = NX * NY - s;           // Body, Eq. (8b)
+}
+
+// Listing 3 compares per region under short-circuit evaluation (A18), Eq. (4) order.
+const int kNSwitch[9] = {2, 3, 3, 6, 8, 8, 8, 9, 8};
+
+// Eqs. (3)-(6), (9), (10).
+void model(const Plan &p, int w, int h, int mw, int mh, const isp_model_params &mp, isp_plan_info &o)
+{
+    const double m = mw, n = mh, c = mp.n_check, k = mp.n_kernel;
+    o.n_naive = (4 * c + k) * m * n * (double)w * h;             // Eq. (3), reading A13
+    if (p.degenerate) {
+        o.n_isp = INFINITY;
+        o.r_reduced = 0;
+        o.g = 0;
+        return;
+    }
+    const double threads = 32.0 * p.wx, pix = (double)p.tile_w * p.ty;
+    double nisp = 0;
+    for (int r = 0; r < 9; ++r) {
+        const double nreg = (r == 0 || r == 1 || r == 3 || r == 4) ? 2 * c + k : (r == 8 ? k : c + k);
+        const double nsw = kNSwitch[r] * mp.ipc_switch;
+        if (mp.form == 1) nisp += (nsw + nreg) * m * n * (double)o.n_block[r] * pix;          // printed
+        else nisp += (nsw * threads + nreg * m * n * pix) * (double)o.n_block[r];             // A14 form T
+    }
+    o.n_isp = nisp;
+    o.r_reduced = o.n_naive / nisp;                                  // Eq. (9)
+    o.g = o.r_reduced * o.o_isp / o.o_naive;                         // Eq. (10)
+}
+
+double occupancy(const void *fn, int threads)
+{
+    if (!fn) return 0;
+    int nb = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, fn, threads, 0) != cudaSuccess) {
+        cudaGetLastError();
+        return 0;
+    }
+    return std::min(1.0, nb * (threads / 32.0) / 64.0);  // 64 warps per SM on sm_100 (A20)
+}
+
+enum Family { F_CONV_F32 = 0, F_SEP_F32 = 1, F_U8 = 2, F_SOBEL = 3, F_LAPLACE = 4, F_HARRIS = 5,
+              F_BILATERAL = 6, F_ATROUS = 7 };
+
+int family_px(int fam, bool direct)
+{
+    if (direct) return PX_DIRECT;
+    switch (fam) {
+    case F_U8: case F_SOBEL: case F_LAPLACE: return PX_U8;
+    case F_HARRIS: return PX_I16;
+    default: return PX_F32;
+    }
+}
+
+void defaults(int fam, int mode, isp_model_params &mp)
+{
+    // Calibration constants: instructions per border check per
+    // tap (mode-dependent) and per tap of the kernel computation.
+    static const double chk[4] = {1.0, 2.0, 3.0, 2.0};
+    mp.n_check = chk[mode & 3];
+    mp.n_kernel = fam == F_BILATERAL ? 8.0 : fam == F_HARRIS ? 3.0 : 1.0;
+    mp.ipc_switch = 2.0;
+    mp.o_naive = -1;
+    mp.o_isp = -1;
+    mp.form = 0;
+}
+
+using KfnFn = const void *(*)(const Desc &);
+using RunFn = cudaError_t (*)(const Desc &);
+
+// Resolve the variant (AUTO = "isp+m") and launch.
+isp_status_t resolve_and_launch(Desc &d, int fam, int w, int h, int mw, int mh, int hx, int hy, bool direct,
+                                isp_variant_t v, KfnFn kfn, RunFn run, const char *what,
+                                const RowRange *rr = nullptr)
+{
+    Plan p = make_plan(w, h, hx, hy, family_px(fam, direct), 0, 0, 0, rr);
+    if (rr) {
+        d.g.oy0 = rr->oy0;
+        d.g.y_end = rr->oy0 + rr->nrows;
+        d.g.ylim = rr->ylim;
+        d.g.t_real = rr->t_real;
+        d.g.b_real = rr->b_real;
+    }
+    d.g.ty = p.ty;
+    d.g.bh_l = p.bh_l;
+    d.g.bh_r = p.bh_r;
+    d.g.bh_t = p.bh_t;
+    d.g.bh_b = p.bh_b;
+    d.g.w_l = p.w_l;
+    d.g.w_r = p.w_r;
+    d.grid = dim3(p.nx, p.ny, 1);
+    d.block = dim3(32 * p.wx, 1, 1);
+    const bool fits = hx <= w && hy <= h;  // one reflection suffices (naive Mirror)
+    const int naive_disp = fits ? DISP_NAIVE : DISP_NAIVE_GEN;
+
+    isp_plan_info info{};
+    info.bh_l = p.bh_l; info.bh_r = p.bh_r; info.bh_t = p.bh_t; info.bh_b = p.bh_b;
+    info.nx = p.nx; info.ny = p.ny; info.w_l = p.w_l; info.w_r = p.w_r;
+    info.degenerate = p.degenerate;
+    info.tile_w = p.tile_w; info.tile_h = p.ty; info.warp_w = p.warp_w;
+    n_block(p, info.n_block);
+
+    isp_variant_t chosen = v;
+    if (p.degenerate) {
+        chosen = ISP_NAIVE;  // A3: Listing 3 cannot express a block needing opposite checks
+    } else if (v == ISP_AUTO) {
+        isp_model_params mp;
+        defaults(fam, d.mode, mp);
+        Desc q = d;
+        q.disp = naive_disp;
+        info.o_naive = occupancy(kfn(q), 32 * p.wx);
+        q.disp = p.wx > 1 ? DISP_WARP : DISP_BLOCK;
+        info.o_isp = occupancy(kfn(q), 32 * p.wx);
+        if (info.o_naive <= 0) info.o_naive = 1;
+        if (info.o_isp <= 0) info.o_isp = 1;
+        model(p, w, h, mw, mh, mp, info);
+        chosen = info.g > 1.0 ? (p.wx > 1 ? ISP_WARP : ISP_BLOCK) : ISP_NAIVE;
+    }
+    info.choice = chosen;
+    d.disp = chosen == ISP_WARP ? DISP_WARP : chosen == ISP_BLOCK ? DISP_BLOCK : naive_disp;
+    g_last_plan = info;
+    cudaError_t e = run(d);
+    if (e == cudaSuccess) e = cudaGetLastError();
+    return cuda_status(e, what);
+}
+
+Desc base_desc(int w, int h, int pitch, int out_pitch, int mode, isp_stream_t stream)
+{
+    Desc d{};
+    d.g.w = w;
+    d.g.h = h;
+    d.g.in_pitch = pitch;
+    d.g.out_pitch = out_pitch;
+    d.g.oy0 = 0;
+    d.g.y_end = h;
+    d.g.ylim = h;
+    d.g.t_real = 1;
+    d.g.b_real = 1;
+    d.mode = mode;
+    d.stream = (cudaStream_t)stream;
+    return d;
+}
+
+bool aligned(const void *p, long long pitch_bytes, int vbytes)
+{
+    return ((uintptr_t)p % vbytes) == 0 && (pitch_bytes % vbytes) == 0;
+}
+
+// exact rank-1 test of a float mask: mask[j][i] == col[j] * row[i]
+bool separable_f32(const float *mask, int mw, int mh, std::vector<float> &row, std::vector<float> &col)
+{
+    int j0 = 0, i0 = 0;
+    float best = 0;
+    for (int j = 0; j < mh; ++j)
+        for (int i = 0; i < mw; ++i)
+            if (std::fabs(mask[j * mw + i]) > best) { best = std::fabs(mask[j * mw + i]); j0 = j; i0 = i; }
+    if (best == 0) return false;
+    row.assign(mask + j0 * mw, mask + j0 * mw + mw);
+    col.resize(mh);
+    for (int j = 0; j < mh; ++j) col[j] = mask[j * mw + i0] / mask[j0 * mw + i0];
+    for (int j = 0; j < mh; ++j)
+        for (int i = 0; i < mw; ++i)
+            if (std::fabs(col[j] * row[i] - mask[j * mw + i]) > 1e-6f * best) return false;
+    return true;
+}
+
+long long gcdll(long long a, long long b)
+{
+    a = a < 0 ? -a : a;
+    b = b < 0 ? -b : b;
+    while (b) { long long t = a % b; a = b; b = t; }
+    return a;
+}
+
+// exact integer rank-1 decomposition mask = col (x) row
+bool separable_i32(const int32_t *mask, int mw, int mh, std::vector<int> &row, std::vector<int> &col)
+{
+    int j0 = -1;
+    for (int j = 0; j < mh && j0 < 0; ++j)
+        for (int i = 0; i < mw; ++i)
+            if (mask[j * mw + i] != 0) { j0 = j; break; }
+    if (j0 < 0) return false;
+    long long g = 0;
+    for (int i = 0; i < mw; ++i) g = gcdll(g, mask[j0 * mw + i]);
+    row.resize(mw);
+    for (int i = 0; i < mw; ++i) row[i] = (int)(mask[j0 * mw + i] / g);
+    int i0 = 0;
+    while (row[i0] == 0) ++i0;
+    col.resize(mh);
+    for (int j = 0; j < mh; ++j) {
+        if (mask[j * mw + i0] % row[i0] != 0) return false;
+        col[j] = mask[j * mw + i0] / row[i0];
+    }
+    for (int j = 0; j < mh; ++j)
+        for (int i = 0; i < mw; ++i)
+            if ((long long)col[j] * row[i] != mask[j * mw + i]) return false;
+    return true;
+}
+
+U8RoundH make_round(int divisor)
+{
+    U8RoundH r{divisor, -1, 0};
+    if (divisor > 0 && (divisor & (divisor - 1)) == 0) {
+        int s = 0;
+        while ((1 << s) < divisor) ++s;
+        r.shift = s;
+        r.half = divisor >> 1;
+    }
+    return r;
+}
+
+}  // namespace
+
+// =====================================================================================
+extern "C" {
+
+const char *isp_status_string(isp_status_t s)
+{
+    switch (s) {
+    case ISP_OK: return "ISP_OK";
+    case ISP_EINVAL: return "ISP_EINVAL";
+    case ISP_EUNSUPPORTED: return "ISP_EUNSUPPORTED";
+    case ISP_EALIAS: return "ISP_EALIAS";
+    case ISP_ECUDA: return "ISP_ECUDA";
+    case ISP_ENCCL: return "ISP_ENCCL";
+    }
+    return "ISP_?";
+}
+
+const char *isp_last_error(void) { return g_err; }
+int isp_version(void) { return 1; }
+
+isp_status_t isp_last_plan(isp_plan_info *out)
+{
+    if (!out) return fail(ISP_EINVAL, "null output");
+    *out = g_last_plan;
+    return ISP_OK;
+}
+
+// Launch-shape override for tuning sweeps (0 = planner default).  Not thread-safe.
+isp_status_t isp_set_launch_override(int warps_x, int tile_h)
+{
+    if (warps_x < 0 || warps_x > 8 || tile_h < 0 || tile_h > 4096) return fail(ISP_EINVAL, "override");
+    g_override_wx = warps_x;
+    g_override_ty = tile_h;
+    return ISP_OK;
+}
+
+}  // extern "C"
+
+// Internal row-range entry points (multi-GPU strips, shard.cu).  `img` is addressed
+// with global rows; `out` points at the output row rr->oy0.
+isp_status_t ispi_filter_f32(const float *img, int w, int h, int pitch, const float *mask, int mw, int mh,
+                             int border_mode, float const_val, float *out, int out_pitch, isp_variant_t variant,
+                             isp_stream_t stream, const RowRange *rr)
+{
+    isp_status_t s = check_geom(w, h, pitch, out_pitch, mw, mh, border_mode);
+    if (s != ISP_OK) return s;
+    if (!img || !out || !mask) return fail(ISP_EINVAL, "null pointer");
+    if (!rr && ranges_overlap(img, img_bytes(w, h, pitch, 4), out, img_bytes(w, h, out_pitch, 4)))
+        return fail(ISP_EALIAS, "input and output overlap");
+    Desc d = base_desc(w, h, pitch, out_pitch, border_mode, stream);
+    d.in0 = img;
+    d.out0 = out;
+    d.cval_f = const_val;
+    d.mw = mw;
+    d.mh = mh;
+    d.g.vec_in = aligned(img, (long long)pitch * 4, 16);
+    d.g.vec_out = aligned(out, (long long)out_pitch * 4, 16);
+    std::vector<float> row, col;
+    if (mw == mh && (mw == 3 || mw == 5 || mw == 7)) {
+        if (separable_f32(mask, mw, mh, row, col)) {
+            d.rowf = row.data();
+            d.colf = col.data();
+            return resolve_and_launch(d, F_SEP_F32, w, h, mw, mh, mw / 2, mh / 2, false, variant, kfn_sep_f32,
+                                      run_sep_f32, "isp_filter(separable)", rr);
+        }
+        d.maskf = mask;
+        return resolve_and_launch(d, F_CONV_F32, w, h, mw, mh, mw / 2, mh / 2, false, variant, kfn_conv_f32,
+                                  run_conv_f32, "isp_filter", rr);
+    }
+    d.maskf = mask;
+    return resolve_and_launch(d, F_CONV_F32, w, h, mw, mh, mw / 2, mh / 2, true, variant, kfn_dconv_f32,
+                              run_dconv_f32, "isp_filter(direct)", rr);
+}
+
+isp_status_t ispi_filter_u8(const uint8_t *img, int w, int h, int pitch, const int32_t *mask, int mw, int mh,
+                            int32_t divisor, int border_mode, int const_val, uint8_t *out, int out_pitch,
+                            isp_variant_t variant, isp_stream_t stream, const RowRange *rr)
+{
+    isp_status_t s = check_geom(w, h, pitch, out_pitch, mw, mh, border_mode);
+    if (s != ISP_OK) return s;
+    if (!img || !out || !mask) return fail(ISP_EINVAL, "null pointer");
+    if (divisor <= 0) return fail(ISP_EINVAL, "divisor %d <= 0", divisor);
+    if (const_val < 0 || const_val > 255) return fail(ISP_EINVAL, "u8 constant %d not in [0,255]", const_val);
+    long long sabs = 0;
+    for (int k = 0; k < mw * mh; ++k) sabs += mask[k] < 0 ? -(long long)mask[k] : mask[k];
+    if (sabs * 255 + divisor >= (1LL << 30)) return fail(ISP_EINVAL, "mask too large for int32 accumulation");
+    if (!rr && ranges_overlap(img, img_bytes(w, h, pitch, 1), out, img_bytes(w, h, out_pitch, 1)))
+        return fail(ISP_EALIAS, "input and output overlap");
+    Desc d = base_desc(w, h, pitch, out_pitch, border_mode, stream);
+    d.in0 = img;
+    d.out0 = out;
+    d.cval_i = const_val;
+    d.mw = mw;
+    d.mh = mh;
+    d.rnd = make_round(divisor);
+    std::vector<int> row, col;
+    if (mw == mh && (mw == 3 || mw == 5 || mw == 7)) {
+        d.g.vec_in = aligned(img, pitch, 8);
+        d.g.vec_out = aligned(out, out_pitch, 8);
+        if (separable_i32(mask, mw, mh, row, col)) {
+            d.rowi = row.data();
+            d.coli = col.data();
+            return resolve_and_launch(d, F_U8, w, h, mw, mh, mw / 2, mh / 2, false, variant, kfn_sep_u8,
+                                      run_sep_u8, "isp_filter_u8(separable)", rr);
+        }
+        d.maski = mask;
+        return resolve_and_launch(d, F_U8, w, h, mw, mh, mw / 2, mh / 2, false, variant, kfn_conv_u8, run_conv_u8,
+                                  "isp_filter_u8", rr);
+    }
+    d.maski = mask;
+    d.g.vec_in = aligned(img, pitch, 4);
+    d.g.vec_out = aligned(out, out_pitch, 4);
+    return resolve_and_launch(d, F_U8, w, h, mw, mh, mw / 2, mh / 2, true, variant, kfn_dconv_u8, run_dconv_u8,
+                              "isp_filter_u8(direct)", rr);
+}
+
+extern "C" {
+
+isp_status_t isp_filter_ex(const float *img, int w, int h, int pitch, const float *mask, int mw, int mh,
+                           int border_mode, float const_val, float *out, int out_pitch, isp_variant_t variant,
+                           isp_stream_t stream)
+{
+    return ispi_filter_f32(img, w, h, pitch, mask, mw, mh, border_mode, const_val, out, out_pitch, variant, stream,
+                           nullptr);
+}
+
+isp_status_t isp_filter(const float *img, int w, int h, int pitch, const float *mask, int mw, int mh,
+                        int border_mode, float const_val, float *out)
+{
+    return isp_filter_ex(img, w, h, pitch, mask, mw, mh, border_mode, const_val, out, pitch, ISP_AUTO, nullptr);
+}
+
+isp_status_t isp_filter_naive(const float *img, int w, int h, int pitch, const float *mask, int mw, int mh,
+                              int border_mode, float const_val, float *out)
+{
+    return isp_filter_ex(img, w, h, pitch, mask, mw, mh, border_mode, const_val, out, pitch, ISP_NAIVE, nullptr);
+}
+
+isp_status_t isp_filter_sep_f32(const float *img, int w, int h, int pitch, const float *row, int mw,
+                                const float *col, int mh, int border_mode, float const_val, float *out,
+                                int out_pitch, isp_variant_t variant, isp_stream_t stream)
+{
+    isp_status_t s = check_geom(w, h, pitch, out_pitch, mw, mh, border_mode);
+    if (s != ISP_OK) return s;
+    if (!img || !out || !row || !col) return fail(ISP_EINVAL, "null pointer");
+    if (ranges_overlap(img, img_bytes(w, h, pitch, 4), out, img_bytes(w, h, out_pitch, 4)))
+        return fail(ISP_EALIAS, "input and output overlap");
+    Desc d = base_desc(w, h, pitch, out_pitch, border_mode, stream);
+    d.in0 = img;
+    d.out0 = out;
+    d.cval_f = const_val;
+    d.mw = mw;
+    d.mh = mh;
+    d.rowf = row;
+    d.colf = col;
+    d.g.vec_in = aligned(img, (long long)pitch * 4, 16);
+    d.g.vec_out = aligned(out, (long long)out_pitch * 4, 16);
+    if (mw == mh && (mw == 3 || mw == 5 || mw == 7))
+        return resolve_and_launch(d, F_SEP_F32, w, h, mw, mh, mw / 2, mh / 2, false, variant, kfn_sep_f32,
+                                  run_sep_f32, "isp_filter_sep_f32");
+    // other windows: the direct family with the outer-product mask
+    std::vector<float> m2((size_t)mw * mh);
+    for (int j = 0; j < mh; ++j)
+        for (int i = 0; i < mw; ++i) m2[j * mw + i] = col[j] * row[i];
+    d.maskf = m2.data();
+    return resolve_and_launch(d, F_SEP_F32, w, h, mw, mh, mw / 2, mh / 2, true, variant, kfn_dconv_f32,
+                              run_dconv_f32, "isp_filter_sep_f32(direct)");
+}
+
+isp_status_t isp_filter_u8(const uint8_t *img, int w, int h, int pitch, const int32_t *mask, int mw, int mh,
+                           int32_t divisor, int border_mode, int const_val, uint8_t *out, int out_pitch,
+                           isp_variant_t variant, isp_stream_t stream)
+{
+    return ispi_filter_u8(img, w, h, pitch, mask, mw, mh, divisor, border_mode, const_val, out, out_pitch, variant,
+                          stream, nullptr);
+}
+
+isp_status_t isp_sobel_u8(const uint8_t *img, int w, int h, int pitch, int border_mode, int const_val,
+                          int16_t *dx, int16_t *dy, uint8_t *mag, int out_pitch, isp_variant_t variant,
+                          isp_stream_t stream)
+{
+    isp_status_t s = check_geom(w, h, pitch, out_pitch, 3, 3, border_mode);
+    if (s != ISP_OK) return s;
+    if (!img || (!dx && !dy && !mag)) return fail(ISP_EINVAL, "null pointer");
+    if (const_val < 0 || const_val > 255) return fail(ISP_EINVAL, "u8 constant %d not in [0,255]", const_val);
+    const size_t ib = img_bytes(w, h, pitch, 1);
+    if ((dx && ranges_overlap(img, ib, dx, img_bytes(w, h, out_pitch, 2))) ||
+        (dy && ranges_overlap(img, ib, dy, img_bytes(w, h, out_pitch, 2))) ||
+        (mag && ranges_overlap(img, ib, mag, img_bytes(w, h, out_pitch, 1))))
+        return fail(ISP_EALIAS, "input and output overlap");
+    Desc d = base_desc(w, h, pitch, out_pitch, border_mode, stream);
+    d.in0 = img;
+    d.out0 = dx;
+    d.out1 = dy;
+    d.out2 = mag;
+    d.cval_i = const_val;
+    d.mw = d.mh = 3;
+    d.g.vec_in = aligned(img, pitch, 8);
+    d.g.vec_out = (!dx || aligned(dx, 2LL * out_pitch, 16)) && (!dy || aligned(dy, 2LL * out_pitch, 16)) &&
+                  (!mag || aligned(mag, out_pitch, 8));
+    return resolve_and_launch(d, F_SOBEL, w, h, 3, 3, 1, 1, false, variant, kfn_sobel, run_sobel, "isp_sobel_u8");
+}
+
+isp_status_t isp_laplace5_u8(const uint8_t *img, int w, int h, int pitch, int border_mode, int const_val,
+                             uint8_t *out, int out_pitch, isp_variant_t variant, isp_stream_t stream)
+{
+    isp_status_t s = check_geom(w, h, pitch, out_pitch, 5, 5, border_mode);
+    if (s != ISP_OK) return s;
+    if (!img || !out) return fail(ISP_EINVAL, "null pointer");
+    if (const_val < 0 || const_val > 255) return fail(ISP_EINVAL, "u8 constant %d not in [0,255]", const_val);
+    if (ranges_overlap(img, img_bytes(w, h, pitch, 1), out, img_bytes(w, h, out_pitch, 1)))
+        return fail(ISP_EALIAS, "input and output overlap");
+    Desc d = base_desc(w, h, pitch, out_pitch, border_mode, stream);
+    d.in0 = img;
+    d.out0 = out;
+    d.cval_i = const_val;
+    d.mw = d.mh = 5;
+    d.g.vec_in = aligned(img, pitch, 8);
+    d.g.vec_out = aligned(out, out_pitch, 8);
+    return resolve_and_launch(d, F_LAPLACE, w, h, 5, 5, 2, 2, false, variant, kfn_laplace5, run_laplace5,
+                              "isp_laplace5_u8");
+}
+
+isp_status_t isp_harris_u8(const int16_t *dx, const int16_t *dy, int w, int h, int pitch, int border_mode,
+                           int const_val, int64_t thr, uint8_t *out, int out_pitch, isp_variant_t variant,
+                           isp_stream_t stream)
+{
+    isp_status_t s = check_geom(w, h, pitch, out_pitch, 3, 3, border_mode);
+    if (s != ISP_OK) return s;
+    if (!dx || !dy || !out) return fail(ISP_EINVAL, "null pointer");
+    if (const_val < -32768 || const_val > 32767) return fail(ISP_EINVAL, "int16 constant %d", const_val);
+    const size_t ob = img_bytes(w, h, out_pitch, 1);
+    if (ranges_overlap(dx, img_bytes(w, h, pitch, 2), out, ob) || ranges_overlap(dy, img_bytes(w, h, pitch, 2), out, ob))
+        return fail(ISP_EALIAS, "input and output overlap");
+    Desc d = base_desc(w, h, pitch, out_pitch, border_mode, stream);
+    d.in0 = dx;
+    d.in1 = dy;
+    d.out0 = out;
+    d.cval_i = const_val;
+    d.thr = thr;
+    d.mw = d.mh = 3;
+    d.g.vec_in = aligned(dx, 2LL * pitch, 8) && aligned(dy, 2LL * pitch, 8);
+    d.g.vec_out = aligned(out, out_pitch, 4);
+    return resolve_and_launch(d, F_HARRIS, w, h, 3, 3, 1, 1, false, variant, kfn_harris, run_harris,
+                              "isp_harris_u8");
+}
+
+isp_status_t isp_bilateral_f32(const float *img, int w, int h, int pitch, int win, float sigma_d, float sigma_r,
+                               int border_mode, float const_val, float *out, int out_pitch, isp_variant_t variant,
+                               isp_stream_t stream)
+{
+    isp_status_t s = check_geom(w, h, pitch, out_pitch, win, win, border_mode);
+    if (s != ISP_OK) return s;
+    if (!img || !out) return fail(ISP_EINVAL, "null pointer");
+    if (!(sigma_d > 0) || !(sigma_r > 0)) return fail(ISP_EINVAL, "sigma must be > 0");
+    if (ranges_overlap(img, img_bytes(w, h, pitch, 4), out, img_bytes(w, h, out_pitch, 4)))
+        return fail(ISP_EALIAS, "input and output overlap");
+    Desc d = base_desc(w, h, pitch, out_pitch, border_mode, stream);
+    d.in0 = img;
+    d.out0 = out;
+    d.cval_f = const_val;
+    d.mw = d.mh = win;
+    const double LOG2E = 1.4426950408889634;
+    d.kr = (float)(-LOG2E / (2.0 * (double)sigma_r * sigma_r));
+    std::vector<float> ls((size_t)win * win);
+    const int hw = win / 2;
+    for (int j = 0; j < win; ++j)
+        for (int i = 0; i < win; ++i) {
+            const double r2 = (double)(i - hw) * (i - hw) + (double)(j - hw) * (j - hw);
+            ls[j * win + i] = (float)(-r2 / (2.0 * (double)sigma_d * sigma_d) * LOG2E);
+        }
+    d.ls = ls.data();
+    d.g.vec_in = 0;
+    d.g.vec_out = aligned(out, (long long)out_pitch * 4, 16);
+    return resolve_and_launch(d, F_BILATERAL, w, h, win, win, hw, hw, true, variant, kfn_bilateral, run_bilateral,
+                              "isp_bilateral_f32");
+}
+
+isp_status_t isp_atrous_f32(const float *img, int w, int h, int pitch, int dilation, int border_mode,
+                            float const_val, int tonemap, float *out, int out_pitch, isp_variant_t variant,
+                            isp_stream_t stream)
+{
+    if (!(dilation == 1 || dilation == 2 || dilation == 4 || dilation == 8))
+        return fail(ISP_EUNSUPPORTED, "dilation %d (built: 1, 2, 4, 8)", dilation);
+    isp_status_t s = check_geom(w, h, pitch, out_pitch, 2 * dilation + 1, 2 * dilation + 1, border_mode);
+    if (s != ISP_OK) return s;
+    if (!img || !out) return fail(ISP_EINVAL, "null pointer");
+    if (ranges_overlap(img, img_bytes(w, h, pitch, 4), out, img_bytes(w, h, out_pitch, 4)))
+        return fail(ISP_EALIAS, "input and output overlap");
+    Desc d = base_desc(w, h, pitch, out_pitch, border_mode, stream);
+    d.in0 = img;
+    d.out0 = out;
+    d.cval_f = const_val;
+    d.mw = d.mh = 2 * dilation + 1;
+    d.dilation = dilation;
+    d.tonemap = tonemap != 0;
+    d.g.vec_in = aligned(img, (long long)pitch * 4, 16);
+    d.g.vec_out = aligned(out, (long long)out_pitch * 4, 16);
+    return resolve_and_launch(d, F_ATROUS, w, h, 3, 3, dilation, dilation, false, variant, kfn_atrous, run_atrous,
+                              "isp_atrous_f32");
+}
+
+isp_status_t isp_night_f32(const float *img, int w, int h, int pitch, int border_mode, float const_val,
+                           float *tmp0, float *tmp1, float *out, int out_pitch, isp_variant_t variant,
+                           isp_stream_t stream)
+{
+    if (!tmp0 || !tmp1) return fail(ISP_EINVAL, "null scratch");
+    isp_status_t s;
+    if ((s = isp_atrous_f32(img, w, h, pitch, 1, border_mode, const_val, 0, tmp0, out_pitch, variant, stream))) return s;
+    if ((s = isp_atrous_f32(tmp0, w, h, out_pitch, 2, border_mode, const_val, 0, tmp1, out_pitch, variant, stream))) return s;
+    if ((s = isp_atrous_f32(tmp1, w, h, out_pitch, 4, border_mode, const_val, 0, tmp0, out_pitch, variant, stream))) return s;
+    return isp_atrous_f32(tmp0, w, h, out_pitch, 8, border_mode, const_val, 1, out, out_pitch, variant, stream);
+}
+
+isp_status_t isp_model_defaults(int filter_id, int border_mode, int mw, int mh, isp_model_params *out)
+{
+    if (!out) return fail(ISP_EINVAL, "null output");
+    (void)mw;
+    (void)mh;
+    defaults(filter_id, border_mode, *out);
+    return ISP_OK;
+}
+
+isp_status_t isp_plan(int w, int h, int mw, int mh, int tile_w, int tile_h, int warp_w, int border_mode,
+                      int filter_id, const isp_model_params *params, isp_plan_info *out)
+{
+    isp_status_t s = check_geom(w, h, w, w, mw, mh, border_mode);
+    if (s != ISP_OK) return s;
+    if (!out) return fail(ISP_EINVAL, "null output");
+    const bool direct = (filter_id == F_BILATERAL) || !((mw == mh) && (mw == 3 || mw == 5 || mw == 7));
+    int hx = mw / 2, hy = mh / 2;
+    Plan p = make_plan(w, h, hx, hy, family_px(filter_id, direct), tile_w, tile_h, warp_w);
+    isp_plan_info info{};
+    info.bh_l = p.bh_l; info.bh_r = p.bh_r; info.bh_t = p.bh_t; info.bh_b = p.bh_b;
+    info.nx = p.nx; info.ny = p.ny; info.w_l = p.w_l; info.w_r = p.w_r;
+    info.degenerate = p.degenerate;
+    info.tile_w = p.tile_w; info.tile_h = p.ty; info.warp_w = p.warp_w;
+    n_block(p, info.n_block);
+    isp_model_params mp;
+    if (params) mp = *params;
+    else defaults(filter_id, border_mode, mp);
+    info.o_naive = mp.o_naive > 0 ? mp.o_naive : 1.0;
+    info.o_isp = mp.o_isp > 0 ? mp.o_isp : 1.0;
+    model(p, w, h, mw, mh, mp, info);
+    info.choice = p.degenerate ? ISP_NAIVE : (info.g > 1.0 ? (p.wx > 1 ? ISP_WARP : ISP_BLOCK) : ISP_NAIVE);
+    *out = info;
+    return ISP_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,18 @@
+// internal.h -- declarations shared by api.cu and shard.cu (not part of the C ABI).
+#pragma once
+#include "../../include/isp.h"
+
+// Output row range of a launch: rows [oy0, oy0+nrows) of an image of height h whose
+// resident input rows end at ylim; t_real / b_real: the range's top / bottom edge is a
+// real image edge (else a strip edge whose neighbour rows arrive by halo exchange).
+struct RowRange {
+    int oy0, nrows, ylim, t_real, b_real;
+};
+
+isp_status_t ispi_fail(isp_status_t s, const char *fmt, ...);
+isp_status_t ispi_filter_f32(const float *img, int w, int h, int pitch, const float *mask, int mw, int mh,
+                             int border_mode, float const_val, float *out, int out_pitch, isp_variant_t variant,
+                             isp_stream_t stream, const RowRange *rr);
+isp_status_t ispi_filter_u8(const uint8_t *img, int w, int h, int pitch, const int32_t *mask, int mw, int mh,
+                            int32_t divisor, int border_mode, int const_val, uint8_t *out, int out_pitch,
+                            isp_variant_t variant, isp_stream_t stream, const RowRange *rr);

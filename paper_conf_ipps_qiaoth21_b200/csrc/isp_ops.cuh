@@ -1,0 +1,450 @@
+// isp_ops.cuh -- the local operators of the paper's evaluation as streaming
+// ops for the region-specialised engine (isp_core.cuh).
+//
+// Each op decomposes its window into a per-input-row horizontal part (hrow) and a
+// vertical accumulation into output-row accumulators (vacc, j = window row), which
+// is exact for integer ops and keeps the f32 generic op's row-major FMA order.
+#pragma once
+#include "isp_core.cuh"
+
+namespace ispk {
+
+template <int PX> struct AccF { float v[PX]; };
+template <int PX, int NC> struct AccI { int v[NC][PX]; };
+
+// ---------------------------------------------------------------------------------
+// Generic f32 local operator, compile-time MW x MH ("Mask").
+// out = sum_j sum_i mask[j][i] * in(x+i-hx, y+j-hy): one FMA chain per output in
+// row-major tap order (j outer, i inner) -- identical in every region / variant.
+// ---------------------------------------------------------------------------------
+template <int MW_, int MH_>
+struct OpConvF32 {
+    using Tin = float;
+    static constexpr int NIN = 1, PX = 4, HX = MW_ / 2, HY = MH_ / 2, MH = MH_, SEGW = PX + 2 * HX;
+    struct Params {
+        Geom g;
+        const float *in[1];
+        float cval;
+        float *out;
+        float mask[MW_ * MH_];
+    };
+    struct H { float s[SEGW]; };
+    using A = AccF<PX>;
+    __host__ __device__ static constexpr bool col_used(int) { return true; }
+    __host__ __device__ static constexpr bool row_used(int) { return true; }
+    __device__ __forceinline__ static void zero(A &a)
+    {
+#pragma unroll
+        for (int e = 0; e < PX; ++e) a.v[e] = 0.f;
+    }
+    __device__ __forceinline__ static void hrow(const Params &, const float (&seg)[1][SEGW], H &h)
+    {
+#pragma unroll
+        for (int k = 0; k < SEGW; ++k) h.s[k] = seg[0][k];
+    }
+    __device__ __forceinline__ static void vacc(const Params &p, int j, const H &h, A &a)
+    {
+#pragma unroll
+        for (int i = 0; i < MW_; ++i)
+#pragma unroll
+            for (int e = 0; e < PX; ++e) a.v[e] = fmaf(p.mask[j * MW_ + i], h.s[e + i], a.v[e]);
+    }
+    template <int CK>
+    __device__ __forceinline__ static void store(const Params &p, const A &a, int x0, int y)
+    {
+        store_px<CK, float, PX>(p.out + (ptrdiff_t)(y - p.g.oy0) * p.g.out_pitch, x0, p.g.w, p.g.vec_out, a.v);
+    }
+};
+
+// ---------------------------------------------------------------------------------
+// Separable f32 operator: row pass then column pass fused per strip (no intermediate
+// image).  h = sum_i row[i] in(x+i-hx, .) ; out = sum_j col[j] h(., y+j-hy).
+// ---------------------------------------------------------------------------------
+template <int MW_, int MH_>
+struct OpSepF32 {
+    using Tin = float;
+    static constexpr int NIN = 1, PX = 4, HX = MW_ / 2, HY = MH_ / 2, MH = MH_, SEGW = PX + 2 * HX;
+    struct Params {
+        Geom g;
+        const float *in[1];
+        float cval;
+        float *out;
+        float row[MW_];
+        float col[MH_];
+    };
+    struct H { float v[PX]; };
+    using A = AccF<PX>;
+    __host__ __device__ static constexpr bool col_used(int) { return true; }
+    __host__ __device__ static constexpr bool row_used(int) { return true; }
+    __device__ __forceinline__ static void zero(A &a)
+    {
+#pragma unroll
+        for (int e = 0; e < PX; ++e) a.v[e] = 0.f;
+    }
+    __device__ __forceinline__ static void hrow(const Params &p, const float (&seg)[1][SEGW], H &h)
+    {
+#pragma unroll
+        for (int e = 0; e < PX; ++e) {
+            float t = p.row[0] * seg[0][e];
+#pragma unroll
+            for (int i = 1; i < MW_; ++i) t = fmaf(p.row[i], seg[0][e + i], t);
+            h.v[e] = t;
+        }
+    }
+    __device__ __forceinline__ static void vacc(const Params &p, int j, const H &h, A &a)
+    {
+#pragma unroll
+        for (int e = 0; e < PX; ++e) a.v[e] = fmaf(p.col[j], h.v[e], a.v[e]);
+    }
+    template <int CK>
+    __device__ __forceinline__ static void store(const Params &p, const A &a, int x0, int y)
+    {
+        store_px<CK, float, PX>(p.out + (ptrdiff_t)(y - p.g.oy0) * p.g.out_pitch, x0, p.g.w, p.g.vec_out, a.v);
+    }
+};
+
+// ---------------------------------------------------------------------------------
+// u8 helpers: round-half-up division and saturation (reading A12).
+// ---------------------------------------------------------------------------------
+struct U8Round {
+    int divisor, shift, half; // shift >= 0: divisor == 1 << shift, half = divisor >> 1
+    __device__ __forceinline__ int operator()(int acc) const
+    {
+        if (shift >= 0) return (acc + half) >> shift;            // floor((acc + d/2) / d)
+        const int num = 2 * acc + divisor, den = 2 * divisor;     // floor((2acc + d) / (2d))
+        int q = num / den;
+        if ((num % den != 0) && (num < 0)) q -= 1;
+        return q;
+    }
+};
+
+__device__ __forceinline__ uint8_t sat_u8(int v) { return (uint8_t)min(255, max(0, v)); }
+
+// Generic u8 local operator with an int32 mask, compile-time MW x MH.
+template <int MW_, int MH_>
+struct OpConvU8 {
+    using Tin = uint8_t;
+    static constexpr int NIN = 1, PX = 8, HX = MW_ / 2, HY = MH_ / 2, MH = MH_, SEGW = PX + 2 * HX;
+    struct Params {
+        Geom g;
+        const uint8_t *in[1];
+        uint8_t cval;
+        uint8_t *out;
+        U8Round rnd;
+        int mask[MW_ * MH_];
+    };
+    struct H { int s[SEGW]; };
+    using A = AccI<PX, 1>;
+    __host__ __device__ static constexpr bool col_used(int) { return true; }
+    __host__ __device__ static constexpr bool row_used(int) { return true; }
+    __device__ __forceinline__ static void zero(A &a)
+    {
+#pragma unroll
+        for (int e = 0; e < PX; ++e) a.v[0][e] = 0;
+    }
+    __device__ __forceinline__ static void hrow(const Params &, const uint8_t (&seg)[1][SEGW], H &h)
+    {
+#pragma unroll
+        for (int k = 0; k < SEGW; ++k) h.s[k] = seg[0][k];
+    }
+    __device__ __forceinline__ static void vacc(const Params &p, int j, const H &h, A &a)
+    {
+#pragma unroll
+        for (int i = 0; i < MW_; ++i)
+#pragma unroll
+            for (int e = 0; e < PX; ++e) a.v[0][e] += p.mask[j * MW_ + i] * h.s[e + i];
+    }
+    template <int CK>
+    __device__ __forceinline__ static void store(const Params &p, const A &a, int x0, int y)
+    {
+        uint8_t o[PX];
+#pragma unroll
+        for (int e = 0; e < PX; ++e) o[e] = sat_u8(p.rnd(a.v[0][e]));
+        store_px<CK, uint8_t, PX>(p.out + (ptrdiff_t)(y - p.g.oy0) * p.g.out_pitch, x0, p.g.w, p.g.vec_out, o);
+    }
+};
+
+// Separable u8 operator with integer row/col weights (exact: integer intermediates).
+template <int MW_, int MH_>
+struct OpSepU8 {
+    using Tin = uint8_t;
+    static constexpr int NIN = 1, PX = 8, HX = MW_ / 2, HY = MH_ / 2, MH = MH_, SEGW = PX + 2 * HX;
+    struct Params {
+        Geom g;
+        const uint8_t *in[1];
+        uint8_t cval;
+        uint8_t *out;
+        U8Round rnd;
+        int row[MW_];
+        int col[MH_];
+    };
+    struct H { int v[PX]; };
+    using A = AccI<PX, 1>;
+    __host__ __device__ static constexpr bool col_used(int) { return true; }
+    __host__ __device__ static constexpr bool row_used(int) { return true; }
+    __device__ __forceinline__ static void zero(A &a)
+    {
+#pragma unroll
+        for (int e = 0; e < PX; ++e) a.v[0][e] = 0;
+    }
+    __device__ __forceinline__ static void hrow(const Params &p, const uint8_t (&seg)[1][SEGW], H &h)
+    {
+#pragma unroll
+        for (int e = 0; e < PX; ++e) {
+            int t = 0;
+#pragma unroll
+            for (int i = 0; i < MW_; ++i) t += p.row[i] * (int)seg[0][e + i];
+            h.v[e] = t;
+        }
+    }
+    __device__ __forceinline__ static void vacc(const Params &p, int j, const H &h, A &a)
+    {
+#pragma unroll
+        for (int e = 0; e < PX; ++e) a.v[0][e] += p.col[j] * h.v[e];
+    }
+    template <int CK>
+    __device__ __forceinline__ static void store(const Params &p, const A &a, int x0, int y)
+    {
+        uint8_t o[PX];
+#pragma unroll
+        for (int e = 0; e < PX; ++e) o[e] = sat_u8(p.rnd(a.v[0][e]));
+        store_px<CK, uint8_t, PX>(p.out + (ptrdiff_t)(y - p.g.oy0) * p.g.out_pitch, x0, p.g.w, p.g.vec_out, o);
+    }
+};
+
+// Exact round-half-up integer square root for n < 2^24 (Sobel magnitude, a9):
+// floor via correctly-rounded sqrtf (n exact in f32) + correction, then +1 iff n - r^2 > r.
+__device__ __forceinline__ int isqrt_round(int n)
+{
+    int r = (int)sqrtf((float)n);
+    if (r * r > n) --r;
+    if ((r + 1) * (r + 1) <= n) ++r;
+    if (n - r * r > r) ++r;
+    return r;
+}
+
+// ---------------------------------------------------------------------------------
+// Sobel: dx = [1,2,1]^T (x) [-1,0,1], dy = [-1,0,1]^T (x) [1,2,1] (correlation,
+// A9), fused with the magnitude point operator.  Exact integers.
+// ---------------------------------------------------------------------------------
+struct OpSobel {
+    using Tin = uint8_t;
+    static constexpr int NIN = 1, PX = 8, HX = 1, HY = 1, MH = 3, SEGW = PX + 2;
+    struct Params {
+        Geom g;
+        const uint8_t *in[1];
+        uint8_t cval;
+        int16_t *dx, *dy;
+        uint8_t *mag;
+    };
+    struct H { int sm[PX], df[PX]; };
+    using A = AccI<PX, 2>;
+    __host__ __device__ static constexpr bool col_used(int) { return true; }
+    __host__ __device__ static constexpr bool row_used(int) { return true; }
+    __device__ __forceinline__ static void zero(A &a)
+    {
+#pragma unroll
+        for (int e = 0; e < PX; ++e) a.v[0][e] = a.v[1][e] = 0;
+    }
+    __device__ __forceinline__ static void hrow(const Params &, const uint8_t (&seg)[1][SEGW], H &h)
+    {
+#pragma unroll
+        for (int e = 0; e < PX; ++e) {
+            const int a = seg[0][e], b = seg[0][e + 1], c = seg[0][e + 2];
+            h.sm[e] = a + 2 * b + c;
+            h.df[e] = c - a;
+        }
+    }
+    __device__ __forceinline__ static void vacc(const Params &, int j, const H &h, A &a)
+    {
+#pragma unroll
+        for (int e = 0; e < PX; ++e) {
+            a.v[0][e] += (j == 1 ? 2 : 1) * h.df[e];
+            if (j != 1) a.v[1][e] += (j - 1) * h.sm[e];
+        }
+    }
+    template <int CK>
+    __device__ __forceinline__ static void store(const Params &p, const A &a, int x0, int y)
+    {
+        const size_t off = (ptrdiff_t)(y - p.g.oy0) * p.g.out_pitch;
+        if (p.dx) {
+            int16_t o[PX];
+#pragma unroll
+            for (int e = 0; e < PX; ++e) o[e] = (int16_t)a.v[0][e];
+            store_px<CK, int16_t, PX>(p.dx + off, x0, p.g.w, p.g.vec_out, o);
+        }
+        if (p.dy) {
+            int16_t o[PX];
+#pragma unroll
+            for (int e = 0; e < PX; ++e) o[e] = (int16_t)a.v[1][e];
+            store_px<CK, int16_t, PX>(p.dy + off, x0, p.g.w, p.g.vec_out, o);
+        }
+        if (p.mag) {
+            uint8_t o[PX];
+#pragma unroll
+            for (int e = 0; e < PX; ++e)
+                o[e] = (uint8_t)min(255, isqrt_round(a.v[0][e] * a.v[0][e] + a.v[1][e] * a.v[1][e]));
+            store_px<CK, uint8_t, PX>(p.mag + off, x0, p.g.w, p.g.vec_out, o);
+        }
+    }
+};
+
+// Laplace 5x5 (a8): box sum minus 25 x centre (== ones mask with centre -24).
+struct OpLaplace5 {
+    using Tin = uint8_t;
+    static constexpr int NIN = 1, PX = 8, HX = 2, HY = 2, MH = 5, SEGW = PX + 4;
+    struct Params {
+        Geom g;
+        const uint8_t *in[1];
+        uint8_t cval;
+        uint8_t *out;
+    };
+    struct H { int box[PX], ctr[PX]; };
+    using A = AccI<PX, 2>;
+    __host__ __device__ static constexpr bool col_used(int) { return true; }
+    __host__ __device__ static constexpr bool row_used(int) { return true; }
+    __device__ __forceinline__ static void zero(A &a)
+    {
+#pragma unroll
+        for (int e = 0; e < PX; ++e) a.v[0][e] = a.v[1][e] = 0;
+    }
+    __device__ __forceinline__ static void hrow(const Params &, const uint8_t (&seg)[1][SEGW], H &h)
+    {
+#pragma unroll
+        for (int e = 0; e < PX; ++e) {
+            int s = 0;
+#pragma unroll
+            for (int i = 0; i < 5; ++i) s += seg[0][e + i];
+            h.box[e] = s;
+            h.ctr[e] = seg[0][e + 2];
+        }
+    }
+    __device__ __forceinline__ static void vacc(const Params &, int j, const H &h, A &a)
+    {
+#pragma unroll
+        for (int e = 0; e < PX; ++e) {
+            a.v[0][e] += h.box[e];
+            if (j == 2) a.v[1][e] = h.ctr[e];
+        }
+    }
+    template <int CK>
+    __device__ __forceinline__ static void store(const Params &p, const A &a, int x0, int y)
+    {
+        uint8_t o[PX];
+#pragma unroll
+        for (int e = 0; e < PX; ++e) o[e] = sat_u8(a.v[0][e] - 25 * a.v[1][e]);
+        store_px<CK, uint8_t, PX>(p.out + (ptrdiff_t)(y - p.g.oy0) * p.g.out_pitch, x0, p.g.w, p.g.vec_out, o);
+    }
+};
+
+// Harris over (dx, dy) int16 (a10; BASELINE configs[2]): 3x3, w = [1,2,1](x)[1,2,1].
+// Sxx, Syy, Sxy < 2^25 fit int32 exactly; R25 in int64.
+struct OpHarris {
+    using Tin = int16_t;
+    static constexpr int NIN = 2, PX = 4, HX = 1, HY = 1, MH = 3, SEGW = PX + 2;
+    struct Params {
+        Geom g;
+        const int16_t *in[2];
+        int16_t cval;
+        long long thr;
+        uint8_t *out;
+    };
+    struct H { int xx[PX], yy[PX], xy[PX]; };
+    using A = AccI<PX, 3>;
+    __host__ __device__ static constexpr bool col_used(int) { return true; }
+    __host__ __device__ static constexpr bool row_used(int) { return true; }
+    __device__ __forceinline__ static void zero(A &a)
+    {
+#pragma unroll
+        for (int e = 0; e < PX; ++e) a.v[0][e] = a.v[1][e] = a.v[2][e] = 0;
+    }
+    __device__ __forceinline__ static void hrow(const Params &, const int16_t (&seg)[2][SEGW], H &h)
+    {
+        int pxx[SEGW], pyy[SEGW], pxy[SEGW];
+#pragma unroll
+        for (int k = 0; k < SEGW; ++k) {
+            const int gx = seg[0][k], gy = seg[1][k];
+            pxx[k] = gx * gx;
+            pyy[k] = gy * gy;
+            pxy[k] = gx * gy;
+        }
+#pragma unroll
+        for (int e = 0; e < PX; ++e) {
+            h.xx[e] = pxx[e] + 2 * pxx[e + 1] + pxx[e + 2];
+            h.yy[e] = pyy[e] + 2 * pyy[e + 1] + pyy[e + 2];
+            h.xy[e] = pxy[e] + 2 * pxy[e + 1] + pxy[e + 2];
+        }
+    }
+    __device__ __forceinline__ static void vacc(const Params &, int j, const H &h, A &a)
+    {
+        const int wj = (j == 1) ? 2 : 1;
+#pragma unroll
+        for (int e = 0; e < PX; ++e) {
+            a.v[0][e] += wj * h.xx[e];
+            a.v[1][e] += wj * h.yy[e];
+            a.v[2][e] += wj * h.xy[e];
+        }
+    }
+    template <int CK>
+    __device__ __forceinline__ static void store(const Params &p, const A &a, int x0, int y)
+    {
+        uint8_t o[PX];
+#pragma unroll
+        for (int e = 0; e < PX; ++e) {
+            const long long sxx = a.v[0][e], syy = a.v[1][e], sxy = a.v[2][e];
+            const long long tr = sxx + syy;
+            const long long r25 = 25 * (sxx * syy - sxy * sxy) - tr * tr;
+            o[e] = r25 > p.thr ? 255 : 0;
+        }
+        store_px<CK, uint8_t, PX>(p.out + (ptrdiff_t)(y - p.g.oy0) * p.g.out_pitch, x0, p.g.w, p.g.vec_out, o);
+    }
+};
+
+// Atrous pass, dilation D (P:L355 Night filter; a12, A26): h = [1,2,1]/4 at taps
+// -D, 0, +D in x and y.  Only the used columns/rows are loaded (sparse window, the
+// "holes"); ISP bounds use the effective half-width D.  Optional fused tone map.
+template <int D>
+struct OpAtrous {
+    using Tin = float;
+    static constexpr int NIN = 1, PX = 4, HX = D, HY = D, MH = 2 * D + 1, SEGW = PX + 2 * D;
+    struct Params {
+        Geom g;
+        const float *in[1];
+        float cval;
+        float *out;
+        int tonemap;
+    };
+    struct H { float v[PX]; };
+    using A = AccF<PX>;
+    __host__ __device__ static constexpr bool col_used(int k)
+    {
+        return k < PX || (k >= D && k < D + PX) || (k >= 2 * D && k < 2 * D + PX);
+    }
+    __host__ __device__ static constexpr bool row_used(int j) { return j == 0 || j == D || j == 2 * D; }
+    __device__ __forceinline__ static void zero(A &a)
+    {
+#pragma unroll
+        for (int e = 0; e < PX; ++e) a.v[e] = 0.f;
+    }
+    __device__ __forceinline__ static void hrow(const Params &, const float (&seg)[1][SEGW], H &h)
+    {
+#pragma unroll
+        for (int e = 0; e < PX; ++e) h.v[e] = fmaf(0.25f, seg[0][e + 2 * D], fmaf(0.5f, seg[0][e + D], 0.25f * seg[0][e]));
+    }
+    __device__ __forceinline__ static void vacc(const Params &, int j, const H &h, A &a)
+    {
+        const float wj = (j == D) ? 0.5f : 0.25f;
+#pragma unroll
+        for (int e = 0; e < PX; ++e) a.v[e] = fmaf(wj, h.v[e], a.v[e]);
+    }
+    template <int CK>
+    __device__ __forceinline__ static void store(const Params &p, const A &a, int x0, int y)
+    {
+        float o[PX];
+#pragma unroll
+        for (int e = 0; e < PX; ++e) o[e] = p.tonemap ? a.v[e] / (1.0f + a.v[e]) : a.v[e];
+        store_px<CK, float, PX>(p.out + (ptrdiff_t)(y - p.g.oy0) * p.g.out_pitch, x0, p.g.w, p.g.vec_out, o);
+    }
+};
+
+}  // namespace ispk

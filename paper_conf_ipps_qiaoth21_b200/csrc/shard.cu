@@ -1,0 +1,220 @@
+// shard.cu -- multi-GPU row strips with an NCCL halo exchange (the
+// paper is single-GPU).  One process per GPU; torch.distributed only
+// bootstraps (broadcast of the ncclUniqueId).
+//
+// Schedule (isp_shard_schedule, pure host, unit-tested on CPU):
+//   rank r owns rows [y0, y0 + strip_h), y0 = r * ceil(H/P);
+//   phase 1 "down": send own bottom hy rows to next, receive the top halo from prev;
+//   phase 2 "up":   send own top hy rows to prev, receive the bottom halo from next;
+//   (prev/next wrap around the ring for Repeat, so no strip has a y border then;
+//   per-pair NCCL ordering matches the two phases, also for P = 2);
+//   launch 0 (no halo needed): the rows not within hy of a halo edge -- overlaps the
+//   exchange; launches 1/2 (after the halo event): the hy rows at each halo edge.
+// Only rank 0 owns the image's T border and rank P-1 its B border (Clamp, Mirror,
+// Constant); interior ranks run only L / Body / R regions.
+#include <cuda_runtime.h>
+#include <nccl.h>
+
+#include <algorithm>
+#include <cstring>
+
+#include "internal.h"
+
+struct isp_shard_ctx {
+    ncclComm_t comm;
+    int rank, nranks, device;
+    cudaEvent_t ev_ready, ev_halo;
+};
+
+namespace {
+
+isp_status_t nccl_status(ncclResult_t r, const char *what)
+{
+    if (r == ncclSuccess) return ISP_OK;
+    return ispi_fail(ISP_ENCCL, "%s: %s", what, ncclGetErrorString(r));
+}
+
+template <class T> ncclDataType_t nccl_type();
+template <> ncclDataType_t nccl_type<float>() { return ncclFloat32; }
+template <> ncclDataType_t nccl_type<uint8_t>() { return ncclUint8; }
+
+template <class T, class F>
+isp_status_t shard_run(isp_shard_ctx *ctx, T *strip, int w, int H, int pitch, int halo, int hy, int mode,
+                       T *out, int out_pitch, cudaStream_t stream, cudaStream_t comm, F &&filter_rows)
+{
+    isp_shard_sched sc;
+    isp_status_t s = isp_shard_schedule(H, ctx->rank, ctx->nranks, halo, hy, mode, &sc);
+    if (s != ISP_OK) return s;
+    if (cudaSetDevice(ctx->device) != cudaSuccess) return ispi_fail(ISP_ECUDA, "cudaSetDevice");
+    const size_t row_elems = (size_t)pitch;
+    if (sc.n_ops > 0) {
+        if (cudaEventRecord(ctx->ev_ready, stream) != cudaSuccess ||
+            cudaStreamWaitEvent(comm, ctx->ev_ready, 0) != cudaSuccess)
+            return ispi_fail(ISP_ECUDA, "event record/wait");
+        if ((s = nccl_status(ncclGroupStart(), "ncclGroupStart")) != ISP_OK) return s;
+        for (int k = 0; k < sc.n_ops; ++k) {
+            const isp_shard_op &op = sc.ops[k];
+            T *buf = strip + (size_t)op.row * row_elems;
+            const size_t cnt = (size_t)op.nrows * row_elems;
+            ncclResult_t r = op.kind == 0 ? ncclSend(buf, cnt, nccl_type<T>(), op.peer, ctx->comm, comm)
+                                          : ncclRecv(buf, cnt, nccl_type<T>(), op.peer, ctx->comm, comm);
+            if (r != ncclSuccess) {
+                ncclGroupEnd();
+                return nccl_status(r, op.kind == 0 ? "ncclSend" : "ncclRecv");
+            }
+        }
+        if ((s = nccl_status(ncclGroupEnd(), "ncclGroupEnd")) != ISP_OK) return s;
+        if (cudaEventRecord(ctx->ev_halo, comm) != cudaSuccess) return ispi_fail(ISP_ECUDA, "event record");
+    }
+    // global-row addressing: buffer row k holds global row y0 - halo + k
+    const T *in_base = strip - ((ptrdiff_t)sc.y0 - halo) * pitch;
+    bool waited = false;
+    for (int k = 0; k < sc.n_launch; ++k) {
+        const isp_shard_launch &L = sc.launch[k];
+        if (L.nrows <= 0) continue;
+        if (L.after_halo && !waited && sc.n_ops > 0) {
+            if (cudaStreamWaitEvent(stream, ctx->ev_halo, 0) != cudaSuccess)
+                return ispi_fail(ISP_ECUDA, "cudaStreamWaitEvent");
+            waited = true;
+        }
+        RowRange rr{L.oy0, L.nrows, L.ylim, L.t_real, L.b_real};
+        T *o = out + ((ptrdiff_t)L.oy0 - sc.y0) * out_pitch;
+        if ((s = filter_rows(in_base, o, rr)) != ISP_OK) return s;
+    }
+    if (sc.n_ops > 0 && !waited && cudaStreamWaitEvent(stream, ctx->ev_halo, 0) != cudaSuccess)
+        return ispi_fail(ISP_ECUDA, "cudaStreamWaitEvent");
+    return ISP_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+isp_status_t isp_shard_rows(int H, int rank, int nranks, int *y0, int *strip_h)
+{
+    if (H < 1 || nranks < 1 || rank < 0 || rank >= nranks || !y0 || !strip_h)
+        return ispi_fail(ISP_EINVAL, "isp_shard_rows(H=%d, rank=%d, nranks=%d)", H, rank, nranks);
+    const long long per = ((long long)H + nranks - 1) / nranks;
+    const long long a = std::min<long long>(H, per * rank), b = std::min<long long>(H, per * (rank + 1));
+    *y0 = (int)a;
+    *strip_h = (int)(b - a);
+    return ISP_OK;
+}
+
+isp_status_t isp_shard_schedule(int H, int rank, int nranks, int halo, int hy, int border_mode,
+                                isp_shard_sched *out)
+{
+    if (!out) return ispi_fail(ISP_EINVAL, "null output");
+    if (border_mode < 0 || border_mode > 3 || hy < 0 || halo < hy)
+        return ispi_fail(ISP_EINVAL, "schedule: mode %d, hy %d, halo %d", border_mode, hy, halo);
+    isp_shard_sched sc;
+    std::memset(&sc, 0, sizeof(sc));
+    isp_status_t s = isp_shard_rows(H, rank, nranks, &sc.y0, &sc.strip_h);
+    if (s != ISP_OK) return s;
+    // every strip must hold its own two halo bands (and feed its neighbours)
+    for (int r = 0; r < nranks; ++r) {
+        int a, b;
+        isp_shard_rows(H, r, nranks, &a, &b);
+        if (nranks > 1 && b < std::max(2 * hy, 1))
+            return ispi_fail(ISP_EINVAL, "strip of rank %d has %d rows < 2*hy = %d", r, b, 2 * hy);
+    }
+    const bool ring = border_mode == ISP_REPEAT && nranks > 1;
+    const int prev = rank > 0 ? rank - 1 : (ring ? nranks - 1 : -1);
+    const int next = rank < nranks - 1 ? rank + 1 : (ring ? 0 : -1);
+    sc.prev = prev;
+    sc.next = next;
+    const int sh = sc.strip_h;
+    if (hy > 0) {
+        // phase 1 (down), phase 2 (up) -- see file header for the per-pair ordering
+        if (next >= 0) sc.ops[sc.n_ops++] = isp_shard_op{0, next, halo + sh - hy, hy};
+        if (prev >= 0) sc.ops[sc.n_ops++] = isp_shard_op{1, prev, halo - hy, hy};
+        if (prev >= 0) sc.ops[sc.n_ops++] = isp_shard_op{0, prev, halo, hy};
+        if (next >= 0) sc.ops[sc.n_ops++] = isp_shard_op{1, next, halo + sh, hy};
+    }
+    const int need_top = prev >= 0 ? hy : 0, need_bot = next >= 0 ? hy : 0;
+    const int t_real = prev < 0, b_real = next < 0;
+    const int y0 = sc.y0;
+    // launch 0: rows that need no halo; reads only own rows (ylim = strip end)
+    sc.launch[sc.n_launch++] = isp_shard_launch{y0 + need_top, sh - need_top - need_bot, y0 + sh, t_real, b_real, 0};
+    if (need_top)
+        sc.launch[sc.n_launch++] = isp_shard_launch{y0, need_top, y0 + sh, 0, 0, 1};
+    if (need_bot)
+        sc.launch[sc.n_launch++] = isp_shard_launch{y0 + sh - need_bot, need_bot, y0 + sh + need_bot, 0, 0, 1};
+    *out = sc;
+    return ISP_OK;
+}
+
+isp_status_t isp_shard_unique_id(unsigned char id[128])
+{
+    if (!id) return ispi_fail(ISP_EINVAL, "null id");
+    ncclUniqueId uid;
+    isp_status_t s = nccl_status(ncclGetUniqueId(&uid), "ncclGetUniqueId");
+    if (s != ISP_OK) return s;
+    static_assert(sizeof(uid.internal) == 128, "ncclUniqueId size");
+    std::memcpy(id, uid.internal, 128);
+    return ISP_OK;
+}
+
+isp_status_t isp_shard_init(isp_shard_ctx **ctx, const unsigned char id[128], int rank, int nranks, int device)
+{
+    if (!ctx || !id || nranks < 1 || rank < 0 || rank >= nranks) return ispi_fail(ISP_EINVAL, "isp_shard_init args");
+    if (cudaSetDevice(device) != cudaSuccess) return ispi_fail(ISP_ECUDA, "cudaSetDevice(%d)", device);
+    isp_shard_ctx *c = new isp_shard_ctx{};
+    c->rank = rank;
+    c->nranks = nranks;
+    c->device = device;
+    ncclUniqueId uid;
+    std::memcpy(uid.internal, id, 128);
+    isp_status_t s = nccl_status(ncclCommInitRank(&c->comm, nranks, uid, rank), "ncclCommInitRank");
+    if (s != ISP_OK) {
+        delete c;
+        return s;
+    }
+    if (cudaEventCreateWithFlags(&c->ev_ready, cudaEventDisableTiming) != cudaSuccess ||
+        cudaEventCreateWithFlags(&c->ev_halo, cudaEventDisableTiming) != cudaSuccess) {
+        ncclCommDestroy(c->comm);
+        delete c;
+        return ispi_fail(ISP_ECUDA, "cudaEventCreate");
+    }
+    *ctx = c;
+    return ISP_OK;
+}
+
+isp_status_t isp_shard_destroy(isp_shard_ctx *ctx)
+{
+    if (!ctx) return ISP_OK;
+    cudaEventDestroy(ctx->ev_ready);
+    cudaEventDestroy(ctx->ev_halo);
+    ncclResult_t r = ncclCommDestroy(ctx->comm);
+    delete ctx;
+    return nccl_status(r, "ncclCommDestroy");
+}
+
+isp_status_t isp_shard_filter_f32(isp_shard_ctx *ctx, float *strip, int w, int H, int pitch, int halo,
+                                  const float *mask, int mw, int mh, int border_mode, float const_val, float *out,
+                                  int out_pitch, isp_variant_t variant, isp_stream_t stream, isp_stream_t comm_stream)
+{
+    if (!ctx || !strip || !out || !mask) return ispi_fail(ISP_EINVAL, "null pointer");
+    auto f = [&](const float *in_base, float *o, const RowRange &rr) {
+        return ispi_filter_f32(in_base, w, H, pitch, mask, mw, mh, border_mode, const_val, o, out_pitch, variant,
+                               stream, &rr);
+    };
+    return shard_run<float>(ctx, strip, w, H, pitch, halo, mh / 2, border_mode, out, out_pitch, (cudaStream_t)stream,
+                            (cudaStream_t)comm_stream, f);
+}
+
+isp_status_t isp_shard_filter_u8(isp_shard_ctx *ctx, uint8_t *strip, int w, int H, int pitch, int halo,
+                                 const int32_t *mask, int mw, int mh, int32_t divisor, int border_mode, int const_val,
+                                 uint8_t *out, int out_pitch, isp_variant_t variant, isp_stream_t stream,
+                                 isp_stream_t comm_stream)
+{
+    if (!ctx || !strip || !out || !mask) return ispi_fail(ISP_EINVAL, "null pointer");
+    auto f = [&](const uint8_t *in_base, uint8_t *o, const RowRange &rr) {
+        return ispi_filter_u8(in_base, w, H, pitch, mask, mw, mh, divisor, border_mode, const_val, o, out_pitch,
+                              variant, stream, &rr);
+    };
+    return shard_run<uint8_t>(ctx, strip, w, H, pitch, halo, mh / 2, border_mode, out, out_pitch,
+                              (cudaStream_t)stream, (cudaStream_t)comm_stream, f);
+}
+
+}  // extern "C"
