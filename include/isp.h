@@ -44,10 +44,14 @@ extern "C" {
 
 typedef enum { ISP_CLAMP = 0, ISP_MIRROR = 1, ISP_REPEAT = 2, ISP_CONSTANT = 3 } isp_border_t;
 typedef enum { ISP_U8 = 0, ISP_I16 = 1, ISP_I32 = 2, ISP_F32 = 3 } isp_dtype_t;
-/* ISP_AUTO = "isp+m": the model of Eq. (10) picks ISP (block or warp
- * granularity) or NAIVE.  ISP_BLOCK = Listing 3; ISP_WARP = Listing 5; ISP_NAIVE =
- * all four checks on every read (Eq. 3 baseline). */
-typedef enum { ISP_AUTO = 0, ISP_BLOCK = 1, ISP_WARP = 2, ISP_NAIVE = 3 } isp_variant_t;
+/* ISP_AUTO = "isp+m": the model of Eq. (10) picks ISP or NAIVE; its ISP is
+ * ISP_TMA where eligible, else ISP_WARP.  ISP_BLOCK = Listing 3 and ISP_WARP = Listing 5
+ * on the register-streaming kernels (per-read checks only where a region needs them);
+ * ISP_TMA = Listing 3 on the TMA-staged kernels (bulk async copies into shared memory;
+ * checks only in the staging of border blocks, reading A21; needs 16-B aligned rows and
+ * a compiled window, else runs as ISP_BLOCK); ISP_NAIVE = all four checks on every read
+ * (Eq. 3 baseline). */
+typedef enum { ISP_AUTO = 0, ISP_BLOCK = 1, ISP_WARP = 2, ISP_NAIVE = 3, ISP_TMA = 4 } isp_variant_t;
 typedef enum {
     ISP_OK = 0,
     ISP_EINVAL = 1,       /* bad size / pitch / window / mode / constant / divisor */

@@ -20,7 +20,7 @@ import os
 import torch
 
 __all__ = [
-    "CLAMP", "MIRROR", "REPEAT", "CONSTANT", "AUTO", "BLOCK", "WARP", "NAIVE", "MODES", "VARIANTS",
+    "CLAMP", "MIRROR", "REPEAT", "CONSTANT", "AUTO", "BLOCK", "WARP", "NAIVE", "TMA", "MODES", "VARIANTS",
     "lib", "IspError", "PlanInfo", "ModelParams",
     "isp_filter", "isp_filter_naive", "isp_filter_ex", "isp_filter_sep_f32", "isp_filter_u8",
     "isp_sobel_u8", "isp_laplace5_u8", "isp_harris_u8", "isp_bilateral_f32", "isp_atrous_f32",
@@ -31,8 +31,8 @@ __all__ = [
 
 CLAMP, MIRROR, REPEAT, CONSTANT = 0, 1, 2, 3
 MODES = {"clamp": CLAMP, "mirror": MIRROR, "repeat": REPEAT, "constant": CONSTANT}
-AUTO, BLOCK, WARP, NAIVE = 0, 1, 2, 3
-VARIANTS = {"auto": AUTO, "block": BLOCK, "warp": WARP, "naive": NAIVE}
+AUTO, BLOCK, WARP, NAIVE, TMA = 0, 1, 2, 3, 4
+VARIANTS = {"auto": AUTO, "block": BLOCK, "warp": WARP, "naive": NAIVE, "tma": TMA}
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_HERE, "libisp.so")

@@ -6,6 +6,7 @@
 #include <cmath>
 #include <cstdarg>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <mutex>
 #include <unordered_map>
@@ -75,8 +76,28 @@ struct Plan {
     bool degenerate;
 };
 
+int g_num_sms = 0;
+
+int num_sms()
+{
+    if (g_num_sms <= 0) {
+        int dev = 0, n = 0;
+        if (cudaGetDevice(&dev) == cudaSuccess && cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev) ==
+                                                      cudaSuccess && n > 0)
+            g_num_sms = n;
+        else {
+            cudaGetLastError();
+            g_num_sms = 148;  // B200 (no device visible: pure-host planning)
+        }
+    }
+    return g_num_sms;
+}
+
+constexpr int kMinRowsPerBlock = 8;
+
+// blocks_per_sm: resident blocks of the kernel that will run (occupancy API); 0 = 8.
 Plan make_plan(int w, int h, int hx, int hy, int px, int tile_w_req, int tile_h_req, int warp_w_req,
-               const RowRange *rr = nullptr)
+               const RowRange *rr = nullptr, int blocks_per_sm = 0)
 {
     const RowRange whole{0, h, h, 1, 1};
     if (!rr) rr = &whole;
@@ -91,30 +112,47 @@ Plan make_plan(int w, int h, int hx, int hy, int px, int tile_w_req, int tile_h_
     } else {
         wx = (int)std::min<long long>(4, std::max<long long>(1, ceil_div(w, warp_w)));
     }
-    int ty;
-    if (tile_h_req > 0) ty = tile_h_req;
-    else if (g_override_ty > 0) ty = g_override_ty;
-    else {
-        // enough tiles for >= ~4 waves of 148 SMs x 8 resident blocks, rows >= 8
-        const long long nxl = ceil_div(w, (long long)wx * warp_w);
-        ty = 32;
-        while (ty > 8 && nxl * ceil_div(rr->nrows, ty) < 148LL * 8) ty /= 2;
-    }
     p.wx = wx;
-    p.ty = ty;
     p.warp_w = warp_w;
     p.tile_w = wx * warp_w;
     p.nx = (int)ceil_div(w, p.tile_w);
-    p.ny = (int)ceil_div(rr->nrows, ty);
+    const int nr = rr->nrows;
+    const int ty_req = tile_h_req > 0 ? tile_h_req : g_override_ty;
+    if (ty_req > 0) {
+        // uniform tiles of ty rows: Eq. (2) verbatim in y
+        p.ty = ty_req;
+        p.ny = (int)ceil_div(nr, p.ty);
+    } else {
+        // balanced split: one wave of resident blocks, >= kMinRowsPerBlock rows each
+        const long long slots = (long long)num_sms() * (blocks_per_sm > 0 ? blocks_per_sm : 8);
+        long long nby = std::max<long long>(1, slots / p.nx);
+        nby = std::min<long long>(nby, std::max(1, nr / kMinRowsPerBlock));
+        p.ty = 0;
+        p.ny = (int)nby;
+    }
     p.bh_l = (int)ceil_div(hx, p.tile_w);
     p.bh_r = (int)floor_div(w - hx, p.tile_w);
-    // Eq. (2) in y, relative to the launch's first row oy0; only real image edges count.
-    p.bh_t = rr->t_real ? (int)std::max<long long>(0, ceil_div(hy - rr->oy0, ty)) : 0;
-    const long long safe_end = rr->b_real ? std::min<long long>(rr->oy0 + rr->nrows, (long long)h - hy)
-                                          : rr->oy0 + rr->nrows;
-    p.bh_b = (int)floor_div(safe_end - rr->oy0, ty);
     p.w_l = (int)ceil_div(hx, warp_w);
     p.w_r = (int)floor_div(w - hx, warp_w);
+    // Eq. (2) in y, relative to the launch's first row oy0; only real image edges count.
+    if (p.ty > 0) {
+        p.bh_t = rr->t_real ? (int)std::max<long long>(0, ceil_div(hy - rr->oy0, p.ty)) : 0;
+        const long long safe_end = rr->b_real ? std::min<long long>(rr->oy0 + nr, (long long)h - hy)
+                                              : rr->oy0 + nr;
+        p.bh_b = (int)floor_div(safe_end - rr->oy0, p.ty);
+    } else {
+        // same definition on the balanced split: first block row whose reads stay >= 0,
+        // first block row whose reads reach past the image bottom
+        auto y0_of = [&](long long by) { return rr->oy0 + (by * nr) / p.ny; };
+        int bt = 0;
+        if (rr->t_real)
+            while (bt < p.ny && y0_of(bt) - hy < 0) ++bt;
+        int bb = p.ny;
+        if (rr->b_real)
+            while (bb > 0 && y0_of(bb) + hy > h) --bb;   // y0_of(bb) = end of block bb-1
+        p.bh_t = bt;
+        p.bh_b = bb;
+    }
     p.degenerate = p.bh_l > p.bh_r || p.bh_t > p.bh_b;
     return p;
 }
@@ -162,16 +200,33 @@ void model(const Plan &p, int w, int h, int mw, int mh, const isp_model_params &
     o.g = o.r_reduced * o.o_isp / o.o_naive;                         // Eq. (10)
 }
 
-double occupancy(const void *fn, int threads)
+// Resident blocks per SM of a kernel (occupancy API), cached per (kernel, block size).
+int blocks_per_sm(const void *fn, int threads, size_t smem = 0)
 {
+    static std::mutex mu;
+    static std::unordered_map<const void *, int> cache[9];
     if (!fn) return 0;
-    int nb = 0;
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, fn, threads, 0) != cudaSuccess) {
-        cudaGetLastError();
-        return 0;
+    const int slot = smem ? 0 : std::min(8, threads / 32);
+    {
+        std::lock_guard<std::mutex> lk(mu);
+        auto it = cache[slot].find(fn);
+        if (it != cache[slot].end()) return it->second;
     }
-    return std::min(1.0, nb * (threads / 32.0) / 64.0);  // 64 warps per SM on sm_100 (A20)
+    int nb = 0;
+    if (smem > 48 * 1024 && cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) !=
+                                cudaSuccess)
+        cudaGetLastError();
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, fn, threads, smem) != cudaSuccess) {
+        cudaGetLastError();
+        nb = 0;
+    }
+    std::lock_guard<std::mutex> lk(mu);
+    cache[slot][fn] = nb;
+    return nb;
 }
+
+// Theoretical occupancy O (reading A20): resident warps / 64 warps per SM on sm_100.
+double occupancy_of(int nb, int threads) { return std::min(1.0, nb * (threads / 32.0) / 64.0); }
 
 enum Family { F_CONV_F32 = 0, F_SEP_F32 = 1, F_U8 = 2, F_SOBEL = 3, F_LAPLACE = 4, F_HARRIS = 5,
               F_BILATERAL = 6, F_ATROUS = 7 };
@@ -202,12 +257,49 @@ void defaults(int fam, int mode, isp_model_params &mp)
 using KfnFn = const void *(*)(const Desc &);
 using RunFn = cudaError_t (*)(const Desc &);
 
-// Resolve the variant (AUTO = "isp+m") and launch.
+// TMA-staged family geometry (isp_staged.cuh): 4 compute warps per CTA, tile width
+// 128*PX, halo rounded up to 16 B (HXA) and Eq. (2)'s x bounds taken with HXA and the
+// 16-B aligned width w_al, so every Body CTA's bulk copies are in bounds (A21).
+struct StagedGeom {
+    int hxa, w_al, sw, stages;
+    size_t smem;
+};
+
+StagedGeom staged_geom(int w, int hx, int hy, int px, int esz, int nin)
+{
+    StagedGeom sg{};
+    const int tw = STAGED_WARPS * 32 * px;
+    sg.hxa = (int)(ceil_div((long long)hx * esz, 16) * 16 / esz);
+    sg.w_al = (int)(((long long)w * esz / 16) * 16 / esz);
+    sg.sw = tw + 2 * sg.hxa;
+    const long long mh = 2 * hy + 1;
+    const long long stage_bytes = mh * nin * sg.sw * esz;
+    sg.stages = (int)std::min<long long>(16, std::max<long long>(3, ceil_div(24 * 1024, stage_bytes)));
+    if (const char *e = getenv("ISP_STAGES")) sg.stages = std::max(2, std::min(16, atoi(e)));
+    sg.smem = 256 + (size_t)sg.stages * stage_bytes;
+    return sg;
+}
+
+void apply_staged_bounds(Plan &p, int w, int px, const StagedGeom &sg)
+{
+    p.wx = STAGED_WARPS;
+    p.warp_w = 32 * px;
+    p.tile_w = STAGED_WARPS * 32 * px;
+    p.nx = (int)ceil_div(w, p.tile_w);
+    p.bh_l = (int)ceil_div(sg.hxa, p.tile_w);
+    p.bh_r = (int)floor_div(sg.w_al - sg.hxa, p.tile_w);
+    p.w_l = p.bh_l * STAGED_WARPS;
+    p.w_r = p.bh_r * STAGED_WARPS;
+    p.degenerate = p.bh_l > p.bh_r || p.bh_t > p.bh_b;
+}
+
+// Resolve the variant (AUTO = "isp+m") and launch.  tma_ok: the op has a staged
+// kernel and the input rows are 16-B aligned; esz / nin: input element size / count.
 isp_status_t resolve_and_launch(Desc &d, int fam, int w, int h, int mw, int mh, int hx, int hy, bool direct,
                                 isp_variant_t v, KfnFn kfn, RunFn run, const char *what,
-                                const RowRange *rr = nullptr)
+                                const RowRange *rr = nullptr, bool tma_ok = false, int esz = 4, int nin = 1)
 {
-    Plan p = make_plan(w, h, hx, hy, family_px(fam, direct), 0, 0, 0, rr);
+    const int px = family_px(fam, direct);
     if (rr) {
         d.g.oy0 = rr->oy0;
         d.g.y_end = rr->oy0 + rr->nrows;
@@ -215,6 +307,47 @@ isp_status_t resolve_and_launch(Desc &d, int fam, int w, int h, int mw, int mh, 
         d.g.t_real = rr->t_real;
         d.g.b_real = rr->b_real;
     }
+    const Plan p0 = make_plan(w, h, hx, hy, px, 0, 0, 0, rr, 0);
+    const int threads = 32 * p0.wx;
+    const bool fits = hx <= w && hy <= h;  // one reflection suffices (naive Mirror)
+    const int naive_disp = fits ? DISP_NAIVE : DISP_NAIVE_GEN;
+    auto fn_of = [&](int disp) {
+        Desc q = d;
+        q.disp = disp;
+        return kfn(q);
+    };
+    const StagedGeom sg = staged_geom(w, hx, hy, px, esz, nin);
+    tma_ok = tma_ok && !direct && fn_of(DISP_TMA) != nullptr && g_override_wx == 0;
+    const int nb_naive = blocks_per_sm(fn_of(naive_disp), threads);
+    const int nb_stream = blocks_per_sm(fn_of(p0.wx > 1 ? DISP_WARP : DISP_BLOCK), threads);
+    const int nb_tma = tma_ok ? blocks_per_sm(fn_of(DISP_TMA), STAGED_THREADS, sg.smem) : 0;
+    if (tma_ok && nb_tma <= 0) tma_ok = false;
+
+    isp_variant_t chosen = v;
+    if (chosen == ISP_TMA && !tma_ok) chosen = ISP_BLOCK;      // misaligned / not built: streaming
+    if (v == ISP_AUTO) chosen = tma_ok ? ISP_TMA : (p0.wx > 1 ? ISP_WARP : ISP_BLOCK);
+    auto plan_for = [&](isp_variant_t c) {
+        if (c == ISP_TMA) {
+            Plan q = make_plan(w, h, hx, hy, px, STAGED_WARPS * 32 * px, 0, 0, rr, nb_tma);
+            apply_staged_bounds(q, w, px, sg);
+            return q;
+        }
+        return make_plan(w, h, hx, hy, px, 0, 0, 0, rr, c == ISP_NAIVE ? nb_naive : nb_stream);
+    };
+    Plan p = plan_for(chosen);
+    isp_plan_info info{};
+    if (p.degenerate) chosen = ISP_NAIVE;  // A3: Listing 3 cannot express a block needing opposite checks
+    if (v == ISP_AUTO && !p.degenerate) {
+        isp_model_params mp;
+        defaults(fam, d.mode, mp);
+        info.o_naive = nb_naive > 0 ? occupancy_of(nb_naive, threads) : 1.0;
+        info.o_isp = chosen == ISP_TMA ? occupancy_of(nb_tma, STAGED_THREADS)
+                                       : (nb_stream > 0 ? occupancy_of(nb_stream, threads) : 1.0);
+        n_block(p, info.n_block);
+        model(p, w, h, mw, mh, mp, info);
+        if (!(info.g > 1.0)) chosen = ISP_NAIVE;
+    }
+    if (chosen == ISP_NAIVE) p = plan_for(ISP_NAIVE);
     d.g.ty = p.ty;
     d.g.bh_l = p.bh_l;
     d.g.bh_r = p.bh_r;
@@ -222,36 +355,24 @@ isp_status_t resolve_and_launch(Desc &d, int fam, int w, int h, int mw, int mh, 
     d.g.bh_b = p.bh_b;
     d.g.w_l = p.w_l;
     d.g.w_r = p.w_r;
+    d.g.hxa = sg.hxa;
+    d.g.w_al = sg.w_al;
+    d.g.sw = sg.sw;
+    d.g.stages = sg.stages;
     d.grid = dim3(p.nx, p.ny, 1);
-    d.block = dim3(32 * p.wx, 1, 1);
-    const bool fits = hx <= w && hy <= h;  // one reflection suffices (naive Mirror)
-    const int naive_disp = fits ? DISP_NAIVE : DISP_NAIVE_GEN;
-
-    isp_plan_info info{};
+    d.block = dim3(chosen == ISP_TMA ? STAGED_THREADS : threads, 1, 1);
+    d.smem = chosen == ISP_TMA ? sg.smem : 0;
     info.bh_l = p.bh_l; info.bh_r = p.bh_r; info.bh_t = p.bh_t; info.bh_b = p.bh_b;
     info.nx = p.nx; info.ny = p.ny; info.w_l = p.w_l; info.w_r = p.w_r;
     info.degenerate = p.degenerate;
-    info.tile_w = p.tile_w; info.tile_h = p.ty; info.warp_w = p.warp_w;
+    info.tile_w = p.tile_w; info.tile_h = p.ty > 0 ? p.ty : (int)ceil_div(d.g.y_end - d.g.oy0, p.ny);
+    info.warp_w = p.warp_w;
     n_block(p, info.n_block);
-
-    isp_variant_t chosen = v;
-    if (p.degenerate) {
-        chosen = ISP_NAIVE;  // A3: Listing 3 cannot express a block needing opposite checks
-    } else if (v == ISP_AUTO) {
-        isp_model_params mp;
-        defaults(fam, d.mode, mp);
-        Desc q = d;
-        q.disp = naive_disp;
-        info.o_naive = occupancy(kfn(q), 32 * p.wx);
-        q.disp = p.wx > 1 ? DISP_WARP : DISP_BLOCK;
-        info.o_isp = occupancy(kfn(q), 32 * p.wx);
-        if (info.o_naive <= 0) info.o_naive = 1;
-        if (info.o_isp <= 0) info.o_isp = 1;
-        model(p, w, h, mw, mh, mp, info);
-        chosen = info.g > 1.0 ? (p.wx > 1 ? ISP_WARP : ISP_BLOCK) : ISP_NAIVE;
-    }
     info.choice = chosen;
-    d.disp = chosen == ISP_WARP ? DISP_WARP : chosen == ISP_BLOCK ? DISP_BLOCK : naive_disp;
+    d.disp = chosen == ISP_TMA ? DISP_TMA : chosen == ISP_WARP ? DISP_WARP : chosen == ISP_BLOCK ? DISP_BLOCK
+                                                                                               : naive_disp;
+    d.g.warp_level = chosen == ISP_WARP;
+    if (const char *e = getenv("ISP_DEBUG_STAGED")) d.g.dbg = atoi(e);
     g_last_plan = info;
     cudaError_t e = run(d);
     if (e == cudaSuccess) e = cudaGetLastError();
@@ -407,11 +528,12 @@ isp_status_t ispi_filter_f32(const float *img, int w, int h, int pitch, const fl
             d.rowf = row.data();
             d.colf = col.data();
             return resolve_and_launch(d, F_SEP_F32, w, h, mw, mh, mw / 2, mh / 2, false, variant, kfn_sep_f32,
-                                      run_sep_f32, "isp_filter(separable)", rr);
+                                      run_sep_f32, "isp_filter(separable)", rr,
+                                      aligned(img, (long long)pitch * 4, 16), 4, 1);
         }
         d.maskf = mask;
         return resolve_and_launch(d, F_CONV_F32, w, h, mw, mh, mw / 2, mh / 2, false, variant, kfn_conv_f32,
-                                  run_conv_f32, "isp_filter", rr);
+                                  run_conv_f32, "isp_filter", rr, aligned(img, (long long)pitch * 4, 16), 4, 1);
     }
     d.maskf = mask;
     return resolve_and_launch(d, F_CONV_F32, w, h, mw, mh, mw / 2, mh / 2, true, variant, kfn_dconv_f32,
@@ -447,11 +569,11 @@ isp_status_t ispi_filter_u8(const uint8_t *img, int w, int h, int pitch, const i
             d.rowi = row.data();
             d.coli = col.data();
             return resolve_and_launch(d, F_U8, w, h, mw, mh, mw / 2, mh / 2, false, variant, kfn_sep_u8,
-                                      run_sep_u8, "isp_filter_u8(separable)", rr);
+                                      run_sep_u8, "isp_filter_u8(separable)", rr, aligned(img, pitch, 16), 1, 1);
         }
         d.maski = mask;
         return resolve_and_launch(d, F_U8, w, h, mw, mh, mw / 2, mh / 2, false, variant, kfn_conv_u8, run_conv_u8,
-                                  "isp_filter_u8", rr);
+                                  "isp_filter_u8", rr, aligned(img, pitch, 16), 1, 1);
     }
     d.maski = mask;
     d.g.vec_in = aligned(img, pitch, 4);
@@ -503,7 +625,8 @@ isp_status_t isp_filter_sep_f32(const float *img, int w, int h, int pitch, const
     d.g.vec_out = aligned(out, (long long)out_pitch * 4, 16);
     if (mw == mh && (mw == 3 || mw == 5 || mw == 7))
         return resolve_and_launch(d, F_SEP_F32, w, h, mw, mh, mw / 2, mh / 2, false, variant, kfn_sep_f32,
-                                  run_sep_f32, "isp_filter_sep_f32");
+                                  run_sep_f32, "isp_filter_sep_f32", nullptr,
+                                  aligned(img, (long long)pitch * 4, 16), 4, 1);
     // other windows: the direct family with the outer-product mask
     std::vector<float> m2((size_t)mw * mh);
     for (int j = 0; j < mh; ++j)
@@ -544,7 +667,8 @@ isp_status_t isp_sobel_u8(const uint8_t *img, int w, int h, int pitch, int borde
     d.g.vec_in = aligned(img, pitch, 8);
     d.g.vec_out = (!dx || aligned(dx, 2LL * out_pitch, 16)) && (!dy || aligned(dy, 2LL * out_pitch, 16)) &&
                   (!mag || aligned(mag, out_pitch, 8));
-    return resolve_and_launch(d, F_SOBEL, w, h, 3, 3, 1, 1, false, variant, kfn_sobel, run_sobel, "isp_sobel_u8");
+    return resolve_and_launch(d, F_SOBEL, w, h, 3, 3, 1, 1, false, variant, kfn_sobel, run_sobel, "isp_sobel_u8",
+                              nullptr, aligned(img, pitch, 16), 1, 1);
 }
 
 isp_status_t isp_laplace5_u8(const uint8_t *img, int w, int h, int pitch, int border_mode, int const_val,
@@ -564,7 +688,7 @@ isp_status_t isp_laplace5_u8(const uint8_t *img, int w, int h, int pitch, int bo
     d.g.vec_in = aligned(img, pitch, 8);
     d.g.vec_out = aligned(out, out_pitch, 8);
     return resolve_and_launch(d, F_LAPLACE, w, h, 5, 5, 2, 2, false, variant, kfn_laplace5, run_laplace5,
-                              "isp_laplace5_u8");
+                              "isp_laplace5_u8", nullptr, aligned(img, pitch, 16), 1, 1);
 }
 
 isp_status_t isp_harris_u8(const int16_t *dx, const int16_t *dy, int w, int h, int pitch, int border_mode,
@@ -588,7 +712,8 @@ isp_status_t isp_harris_u8(const int16_t *dx, const int16_t *dy, int w, int h, i
     d.g.vec_in = aligned(dx, 2LL * pitch, 8) && aligned(dy, 2LL * pitch, 8);
     d.g.vec_out = aligned(out, out_pitch, 4);
     return resolve_and_launch(d, F_HARRIS, w, h, 3, 3, 1, 1, false, variant, kfn_harris, run_harris,
-                              "isp_harris_u8");
+                              "isp_harris_u8", nullptr,
+                              aligned(dx, 2LL * pitch, 16) && aligned(dy, 2LL * pitch, 16), 2, 2);
 }
 
 isp_status_t isp_bilateral_f32(const float *img, int w, int h, int pitch, int win, float sigma_d, float sigma_r,

@@ -26,16 +26,14 @@ __device__ __forceinline__ T load_x(const T *__restrict__ row, bool rowok, int x
 }
 
 template <class Op, int MODE, int CK>
-__device__ __forceinline__ void direct_body(const typename Op::Params &p, int x0, int y0)
+__device__ __forceinline__ void direct_body(const typename Op::Params &p, int x0, int y0, int rows)
 {
     using T = typename Op::Tin;
     constexpr int PX = Op::PX;
-    constexpr bool GEN = (CK & CK_GEN) != 0;
     const Geom &g = p.g;
     const int hx = p.mw / 2, hy = p.mh / 2;
-    for (int o = 0; o < g.ty; ++o) {
+    for (int o = 0; o < rows; ++o) {
         const int y = y0 + o;
-        if ((CK & CK_B) && y >= g.y_end) break;
         typename Op::A acc;
         Op::init(p, acc, x0, y);
         for (int j = 0; j < p.mh; ++j) {
@@ -66,23 +64,24 @@ __global__ void __launch_bounds__(256) k_direct(const __grid_constant__ typename
     const int bx = blockIdx.x, by = blockIdx.y;
     const int gw = bx * nwarp + warp;
     const int x0 = (gw * 32 + lane) * Op::PX;
-    const int y0 = p.g.oy0 + by * p.g.ty;
+    int y0, rows;
+    block_rows(p.g, by, gridDim.y, y0, rows);
     if constexpr (DISP == DISP_NAIVE) {
-        direct_body<Op, MODE, CK_ALL>(p, x0, y0);
+        direct_body<Op, MODE, CK_ALL>(p, x0, y0, rows);
     } else if constexpr (DISP == DISP_NAIVE_GEN) {
-        direct_body<Op, MODE, CK_ALL | CK_GEN>(p, x0, y0);
+        direct_body<Op, MODE, CK_ALL | CK_GEN>(p, x0, y0, rows);
     } else {
-        const int rg = region_of(p.g, bx, by, gw, DISP == DISP_WARP);
+        const int rg = region_of(p.g, bx, by, gw, p.g.warp_level != 0);
         switch (rg) {
-        case RG_TL: direct_body<Op, MODE, region_checks(RG_TL)>(p, x0, y0); break;
-        case RG_TR: direct_body<Op, MODE, region_checks(RG_TR)>(p, x0, y0); break;
-        case RG_T: direct_body<Op, MODE, region_checks(RG_T)>(p, x0, y0); break;
-        case RG_BL: direct_body<Op, MODE, region_checks(RG_BL)>(p, x0, y0); break;
-        case RG_BR: direct_body<Op, MODE, region_checks(RG_BR)>(p, x0, y0); break;
-        case RG_B: direct_body<Op, MODE, region_checks(RG_B)>(p, x0, y0); break;
-        case RG_R: direct_body<Op, MODE, region_checks(RG_R)>(p, x0, y0); break;
-        case RG_L: direct_body<Op, MODE, region_checks(RG_L)>(p, x0, y0); break;
-        default: direct_body<Op, MODE, 0>(p, x0, y0); break;
+        case RG_TL: direct_body<Op, MODE, region_checks(RG_TL)>(p, x0, y0, rows); break;
+        case RG_TR: direct_body<Op, MODE, region_checks(RG_TR)>(p, x0, y0, rows); break;
+        case RG_T: direct_body<Op, MODE, region_checks(RG_T)>(p, x0, y0, rows); break;
+        case RG_BL: direct_body<Op, MODE, region_checks(RG_BL)>(p, x0, y0, rows); break;
+        case RG_BR: direct_body<Op, MODE, region_checks(RG_BR)>(p, x0, y0, rows); break;
+        case RG_B: direct_body<Op, MODE, region_checks(RG_B)>(p, x0, y0, rows); break;
+        case RG_R: direct_body<Op, MODE, region_checks(RG_R)>(p, x0, y0, rows); break;
+        case RG_L: direct_body<Op, MODE, region_checks(RG_L)>(p, x0, y0, rows); break;
+        default: direct_body<Op, MODE, 0>(p, x0, y0, rows); break;
         }
     }
 }

@@ -21,6 +21,8 @@ template <int MW_, int MH_>
 struct OpConvF32 {
     using Tin = float;
     static constexpr int NIN = 1, PX = 4, HX = MW_ / 2, HY = MH_ / 2, MH = MH_, SEGW = PX + 2 * HX;
+    static constexpr int PFMAX = 1;
+    static constexpr bool ROW_DIRECT = false;
     struct Params {
         Geom g;
         const float *in[1];
@@ -64,6 +66,8 @@ template <int MW_, int MH_>
 struct OpSepF32 {
     using Tin = float;
     static constexpr int NIN = 1, PX = 4, HX = MW_ / 2, HY = MH_ / 2, MH = MH_, SEGW = PX + 2 * HX;
+    static constexpr int PFMAX = 1;
+    static constexpr bool ROW_DIRECT = false;
     struct Params {
         Geom g;
         const float *in[1];
@@ -125,6 +129,8 @@ template <int MW_, int MH_>
 struct OpConvU8 {
     using Tin = uint8_t;
     static constexpr int NIN = 1, PX = 8, HX = MW_ / 2, HY = MH_ / 2, MH = MH_, SEGW = PX + 2 * HX;
+    static constexpr int PFMAX = 1;
+    static constexpr bool ROW_DIRECT = false;
     struct Params {
         Geom g;
         const uint8_t *in[1];
@@ -169,6 +175,8 @@ template <int MW_, int MH_>
 struct OpSepU8 {
     using Tin = uint8_t;
     static constexpr int NIN = 1, PX = 8, HX = MW_ / 2, HY = MH_ / 2, MH = MH_, SEGW = PX + 2 * HX;
+    static constexpr int PFMAX = 1;
+    static constexpr bool ROW_DIRECT = false;
     struct Params {
         Geom g;
         const uint8_t *in[1];
@@ -230,6 +238,8 @@ __device__ __forceinline__ int isqrt_round(int n)
 struct OpSobel {
     using Tin = uint8_t;
     static constexpr int NIN = 1, PX = 8, HX = 1, HY = 1, MH = 3, SEGW = PX + 2;
+    static constexpr int PFMAX = 1;
+    static constexpr bool ROW_DIRECT = false;
     struct Params {
         Geom g;
         const uint8_t *in[1];
@@ -293,6 +303,8 @@ struct OpSobel {
 struct OpLaplace5 {
     using Tin = uint8_t;
     static constexpr int NIN = 1, PX = 8, HX = 2, HY = 2, MH = 5, SEGW = PX + 4;
+    static constexpr int PFMAX = 1;
+    static constexpr bool ROW_DIRECT = false;
     struct Params {
         Geom g;
         const uint8_t *in[1];
@@ -342,6 +354,8 @@ struct OpLaplace5 {
 struct OpHarris {
     using Tin = int16_t;
     static constexpr int NIN = 2, PX = 4, HX = 1, HY = 1, MH = 3, SEGW = PX + 2;
+    static constexpr int PFMAX = 1;
+    static constexpr bool ROW_DIRECT = false;
     struct Params {
         Geom g;
         const int16_t *in[2];
@@ -407,6 +421,10 @@ template <int D>
 struct OpAtrous {
     using Tin = float;
     static constexpr int NIN = 1, PX = 4, HX = D, HY = D, MH = 2 * D + 1, SEGW = PX + 2 * D;
+    static constexpr int PFMAX = 0;
+    static constexpr bool ROW_DIRECT = true;
+    static constexpr int NTAPS_Y = 3;
+    __host__ __device__ static constexpr int vtap(int t) { return (t - 1) * D; }
     struct Params {
         Geom g;
         const float *in[1];

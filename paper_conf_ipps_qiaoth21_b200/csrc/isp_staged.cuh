@@ -1,0 +1,284 @@
+// isp_staged.cuh -- TMA-staged ISP kernels (bulk async copies + mbarrier pipeline).
+//
+// The B200-native form of the paper's fat kernel: one CTA per block of the
+// partition (Listing 3 on blockIdx), four compute warps plus one producer
+// warp.  The producer streams the CTA's input rows (tile + halo) into a ring of shared
+// memory stages with cp.async.bulk (TMA engine, SASS UBLKCP) completing on mbarriers;
+// the compute warps run the operator from shared memory with no bounds checks at all.
+//
+// Iteration space partitioning moves into the staging (reading A21): a Body CTA's rows
+// and columns are all in bounds, so its producer issues plain bulk copies -- no index
+// arithmetic per pixel; a border CTA maps only its out-of-bounds ROWS (T/B regions,
+// once per row) and fixes up only its out-of-bounds COLUMNS (L/R regions, <= halo
+// elements per row) through the border pattern.  The arithmetic the
+// compute warps execute is identical to the streaming family (same op, same order),
+// so results are bitwise identical to ISP_BLOCK / ISP_WARP / ISP_NAIVE.
+#pragma once
+#include "isp_ops.cuh"
+
+namespace ispk {
+
+constexpr int kStagedComputeWarps = 4;
+constexpr int kStagedThreads = 32 * (kStagedComputeWarps + 1);
+constexpr int kStagedBarrierBytes = 256;  // full[16] + empty[16] mbarriers
+
+__device__ __forceinline__ uint32_t smem_u32(const void *p) { return (uint32_t)__cvta_generic_to_shared(p); }
+
+__device__ __forceinline__ void mbar_init(uint64_t *b, uint32_t count)
+{
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(b)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t *b, uint32_t bytes)
+{
+    asm volatile("mbarrier.expect_tx.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(b)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t *b)
+{
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(b)) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t *b, uint32_t parity)
+{
+    asm volatile(
+        "{\n\t.reg .pred P1;\n\t"
+        "LAB_WAIT:\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n\t"
+        "@P1 bra DONE;\n\t"
+        "bra LAB_WAIT;\n\t"
+        "DONE:\n\t}" ::"r"(smem_u32(b)),
+        "r"(parity)
+        : "memory");
+}
+__device__ __forceinline__ void bulk_g2s(void *dst, const void *src, uint32_t bytes, uint64_t *bar)
+{
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                     smem_u32(dst)),
+                 "l"(src), "r"(bytes), "r"(smem_u32(bar))
+                 : "memory");
+}
+__device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
+__device__ __forceinline__ void fence_mbar_init() { asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory"); }
+
+template <int N>
+__device__ __forceinline__ void lds_words(uint32_t *dst, const void *src)
+{
+    if constexpr (N == 4) {
+        const uint4 q = *reinterpret_cast<const uint4 *>(src);
+        dst[0] = q.x; dst[1] = q.y; dst[2] = q.z; dst[3] = q.w;
+    } else if constexpr (N == 2) {
+        const uint2 q = *reinterpret_cast<const uint2 *>(src);
+        dst[0] = q.x; dst[1] = q.y;
+    } else {
+        dst[0] = *reinterpret_cast<const uint32_t *>(src);
+    }
+}
+
+// One row segment from shared memory: srow points at this thread's column x0.
+template <class Op>
+__device__ __forceinline__ void load_row_smem(const typename Op::Tin *const (&srow)[Op::NIN], RawRow<Op> &rr)
+{
+    using T = typename Op::Tin;
+    using U = VecUse<Op>;
+    constexpr int PX = Op::PX, NV = RawRow<Op>::NV, WPV = U::WPV;
+#pragma unroll
+    for (int c = 0; c < Op::NIN; ++c)
+#pragma unroll
+        for (int v = -NV; v <= NV; ++v) {
+            if (U::lo(v) >= PX) continue;
+            uint32_t(&wv)[WPV] = rr.w[c][v + NV];
+            const int fw = U::first_word(v), n = U::nwords(v);
+            const char *src = reinterpret_cast<const char *>(srow[c] + v * PX) + 4 * fw;
+            if constexpr (WPV >= 4) {
+                if (n == 4) { lds_words<4>(&wv[fw], src); continue; }
+            }
+            if constexpr (WPV >= 2) {
+                if (n == 2) { lds_words<2>(&wv[fw], src); continue; }
+            }
+            lds_words<1>(&wv[fw], src);
+        }
+}
+
+// Value of global column x of a row that needs a fix-up (x outside the bulk-copied
+// range): in-bounds tail, border pattern, or don't-care beyond the window's reach.
+template <class Op, int MODE, int CK>
+__device__ __forceinline__ typename Op::Tin fixup_value(const typename Op::Tin *__restrict__ src, int x,
+                                                        const Geom &g, typename Op::Tin cval)
+{
+    using T = typename Op::Tin;
+    if (x >= 0 && x < g.w) return __ldg(src + x);
+    if (x < -Op::HX || x >= g.w + Op::HX) return T(0);  // no stored output reads it
+    if constexpr (MODE == CONSTANT) {
+        return cval;
+    } else {
+        if constexpr ((CK & CK_L) != 0) {
+            if (x < 0) return __ldg(src + bmap<MODE, true, false, false>(x, g.w));
+        }
+        if constexpr ((CK & CK_R) != 0) {
+            if (x >= g.w) return __ldg(src + bmap<MODE, false, true, false>(x, g.w));
+        }
+        return T(0);
+    }
+}
+
+template <class Op, int MODE, int CK>
+__device__ __forceinline__ void staged_body(const typename Op::Params &p, unsigned char *smem)
+{
+    using T = typename Op::Tin;
+    constexpr int MH = Op::MH, HY = Op::HY, PX = Op::PX, NIN = Op::NIN, SEGW = PX + 2 * Op::HX;
+    constexpr int NWC = kStagedComputeWarps, TW = NWC * 32 * PX;
+    const Geom &g = p.g;
+    const int S = g.stages, SW = g.sw, HXA = g.hxa;
+    uint64_t *full = reinterpret_cast<uint64_t *>(smem);
+    uint64_t *empty = full + 16;
+    T *buf = reinterpret_cast<T *>(smem + kStagedBarrierBytes);
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    int y0, rows;
+    block_rows(g, blockIdx.y, gridDim.y, y0, rows);
+    const int nr = rows + 2 * HY;
+    const int nfill = (nr + MH - 1) / MH;
+    const int X0 = blockIdx.x * TW;          // first output column of the CTA
+    const int XS = X0 - HXA;                 // global column of smem column 0
+    const size_t stage_elems = (size_t)MH * NIN * SW;
+
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < S; ++s) {
+            mbar_init(&full[s], 1);
+            mbar_init(&empty[s], NWC);
+        }
+        fence_mbar_init();
+    }
+    __syncthreads();
+
+    if (warp == NWC) {
+        // ---------------- producer warp ----------------
+        for (int i = 0; i < nfill; ++i) {
+            const int s = i % S;
+            if (i >= S) mbar_wait(&empty[s], ((i / S) - 1) & 1);
+            T *sb = buf + (size_t)s * stage_elems;
+            int yyk[MH], csk[MH], cek[MH];
+            bool okk[MH];
+            uint32_t bytes = 0;
+#pragma unroll
+            for (int k = 0; k < MH; ++k) {
+                const int r = i * MH + k;
+                bool rowok = false;
+                int yy = 0, cs = 0, ce = 0;
+                if (r < nr) {
+                    yy = map_row<MODE, CK>(y0 - HY + r, g, rowok);
+                    cs = XS;
+                    ce = X0 + TW + HXA;
+                    if constexpr ((CK & CK_L) != 0) cs = max(cs, 0);
+                    if constexpr ((CK & CK_R) != 0) ce = min(ce, g.w_al);
+                    if (MODE == CONSTANT && !rowok) ce = cs;  // whole row = C
+                    if (ce > cs) bytes += (uint32_t)(ce - cs) * (uint32_t)sizeof(T) * NIN;
+                }
+                yyk[k] = yy;
+                okk[k] = (r < nr) && (MODE != CONSTANT || rowok);
+                csk[k] = cs;
+                cek[k] = ce;
+            }
+            if (lane == 0) {
+                mbar_expect_tx(&full[s], bytes);
+#pragma unroll
+                for (int k = 0; k < MH; ++k)
+                    if (cek[k] > csk[k])
+#pragma unroll
+                        for (int c = 0; c < NIN; ++c)
+                            bulk_g2s(sb + ((size_t)k * NIN + c) * SW + (csk[k] - XS),
+                                     p.in[c] + (ptrdiff_t)yyk[k] * g.in_pitch + csk[k],
+                                     (uint32_t)(cek[k] - csk[k]) * (uint32_t)sizeof(T), &full[s]);
+            }
+            if constexpr (CK != 0) {
+                // border fix-ups (this region's sides only): generic stores by the warp
+#pragma unroll
+                for (int k = 0; k < MH; ++k) {
+                    const int r = i * MH + k;
+                    if (r >= nr) continue;
+#pragma unroll
+                    for (int c = 0; c < NIN; ++c) {
+                        T *dst = sb + ((size_t)k * NIN + c) * SW;
+                        if (MODE == CONSTANT && !okk[k]) {
+                            for (int x = lane; x < SW; x += 32) dst[x] = p.cval;
+                            continue;
+                        }
+                        const T *src = p.in[c] + (ptrdiff_t)yyk[k] * g.in_pitch;
+                        if constexpr ((CK & CK_L) != 0)
+                            for (int x = XS + lane; x < csk[k]; x += 32)
+                                dst[x - XS] = fixup_value<Op, MODE, CK>(src, x, g, p.cval);
+                        if constexpr ((CK & CK_R) != 0)
+                            for (int x = cek[k] + lane; x < X0 + TW + HXA; x += 32)
+                                dst[x - XS] = fixup_value<Op, MODE, CK>(src, x, g, p.cval);
+                    }
+                }
+                fence_proxy_async();  // order generic writes before later async writes
+            }
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&full[s]);
+        }
+        return;
+    }
+
+    // ---------------- compute warps ----------------
+    const int xoff = (warp * 32 + lane) * PX;  // column within the tile
+    const int x0 = X0 + xoff;
+    typename Op::A acc[MH];
+#pragma unroll
+    for (int k = 0; k < MH; ++k) Op::zero(acc[k]);
+    for (int i = 0; i < nfill; ++i) {
+        const int s = i % S;
+        mbar_wait(&full[s], (i / S) & 1);
+        const T *sb = buf + (size_t)s * stage_elems;
+        if (g.dbg == 1) {
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&empty[s]);
+            continue;
+        }
+#pragma unroll
+        for (int k = 0; k < MH; ++k) {
+            const int r = i * MH + k;
+            if (r < nr) {
+                const T *srow[NIN];
+#pragma unroll
+                for (int c = 0; c < NIN; ++c) srow[c] = sb + ((size_t)k * NIN + c) * SW + HXA + xoff;
+                RawRow<Op> rr;
+                load_row_smem<Op>(srow, rr);
+                T seg[NIN][SEGW];
+                unpack_row<Op>(rr, seg);
+                typename Op::H hs;
+                Op::hrow(p, seg, hs);
+#pragma unroll
+                for (int j = 0; j < MH; ++j) {
+                    if (!Op::row_used(j)) continue;
+                    const int o = r - j;
+                    if (o >= 0 && o < rows) Op::vacc(p, j, hs, acc[(k - j + MH) % MH]);
+                }
+                const int o = r - (MH - 1);
+                if (o >= 0 && g.dbg != 2) Op::template store<CK & CK_R>(p, acc[(k + 1) % MH], x0, y0 + o);
+                Op::zero(acc[(k + 1) % MH]);
+            }
+        }
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&empty[s]);
+    }
+}
+
+// The TMA-staged fat kernel: Listing 3 on (blockIdx.x, blockIdx.y) with the staging
+// bounds of Geom (BH_L/BH_R from the aligned halo HXA, reading A21).
+template <class Op, int MODE>
+__global__ void __launch_bounds__(kStagedThreads) k_staged(const __grid_constant__ typename Op::Params p)
+{
+    extern __shared__ __align__(128) unsigned char smem[];
+    const int rg = region_of(p.g, blockIdx.x, blockIdx.y, 0, false);
+    switch (rg) {
+    case RG_TL: staged_body<Op, MODE, region_checks(RG_TL)>(p, smem); break;
+    case RG_TR: staged_body<Op, MODE, region_checks(RG_TR)>(p, smem); break;
+    case RG_T: staged_body<Op, MODE, region_checks(RG_T)>(p, smem); break;
+    case RG_BL: staged_body<Op, MODE, region_checks(RG_BL)>(p, smem); break;
+    case RG_BR: staged_body<Op, MODE, region_checks(RG_BR)>(p, smem); break;
+    case RG_B: staged_body<Op, MODE, region_checks(RG_B)>(p, smem); break;
+    case RG_R: staged_body<Op, MODE, region_checks(RG_R)>(p, smem); break;
+    case RG_L: staged_body<Op, MODE, region_checks(RG_L)>(p, smem); break;
+    default: staged_body<Op, MODE, 0>(p, smem); break;
+    }
+}
+
+}  // namespace ispk

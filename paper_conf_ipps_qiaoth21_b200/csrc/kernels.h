@@ -18,6 +18,7 @@ struct Desc {
     Geom g;
     int mode, disp;
     dim3 grid, block;
+    size_t smem;  // dynamic shared memory (TMA-staged family)
     cudaStream_t stream;
     const void *in0, *in1;
     void *out0, *out1, *out2;
@@ -61,5 +62,6 @@ cudaError_t run_bilateral(const Desc &);
 
 // pixels per thread (x) of each family
 constexpr int PX_F32 = 4, PX_U8 = 8, PX_I16 = 4, PX_DIRECT = 4;
+constexpr int STAGED_WARPS = 4, STAGED_THREADS = 160;
 
 }  // namespace ispk

@@ -1,7 +1,11 @@
 // launch.cuh -- template glue: pick the (op, mode, dispatch) kernel instance and launch it.
 #pragma once
+#include <mutex>
+#include <unordered_set>
+
 #include "isp_direct.cuh"
 #include "isp_ops.cuh"
+#include "isp_staged.cuh"
 #include "kernels.h"
 
 namespace ispk {
@@ -12,7 +16,7 @@ const void *kernel_for_disp(int disp)
     if constexpr (DIRECT) {
         switch (disp) {
         case DISP_BLOCK: return (const void *)k_direct<Op, MODE, DISP_BLOCK>;
-        case DISP_WARP: return (const void *)k_direct<Op, MODE, DISP_WARP>;
+        case DISP_WARP: return (const void *)k_direct<Op, MODE, DISP_BLOCK>;
         case DISP_NAIVE: return (const void *)k_direct<Op, MODE, DISP_NAIVE>;
         default:
             if constexpr (MODE == MIRROR) return (const void *)k_direct<Op, MODE, DISP_NAIVE_GEN>;
@@ -20,8 +24,11 @@ const void *kernel_for_disp(int disp)
         }
     } else {
         switch (disp) {
+        case DISP_TMA:
+            if constexpr (!Op::ROW_DIRECT) return (const void *)k_staged<Op, MODE>;
+            else return nullptr;
         case DISP_BLOCK: return (const void *)k_stencil<Op, MODE, DISP_BLOCK>;
-        case DISP_WARP: return (const void *)k_stencil<Op, MODE, DISP_WARP>;
+        case DISP_WARP: return (const void *)k_stencil<Op, MODE, DISP_BLOCK>;
         case DISP_NAIVE: return (const void *)k_stencil<Op, MODE, DISP_NAIVE>;
         default:
             if constexpr (MODE == MIRROR) return (const void *)k_stencil<Op, MODE, DISP_NAIVE_GEN>;
@@ -46,8 +53,18 @@ template <class P>
 cudaError_t launch_params(const void *fn, const Desc &d, const P &p)
 {
     if (!fn) return cudaErrorNotSupported;
+    if (d.smem > 48 * 1024) {
+        static std::mutex mu;
+        static std::unordered_set<const void *> done;
+        std::lock_guard<std::mutex> lk(mu);
+        if (!done.count(fn)) {
+            cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)d.smem);
+            if (e != cudaSuccess) return e;
+            done.insert(fn);
+        }
+    }
     void *args[] = {const_cast<P *>(&p)};
-    return cudaLaunchKernel(fn, d.grid, d.block, args, 0, d.stream);
+    return cudaLaunchKernel(fn, d.grid, d.block, args, d.smem, d.stream);
 }
 
 }  // namespace ispk

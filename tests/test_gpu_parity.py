@@ -21,7 +21,7 @@ import synth
 pytestmark = pytest.mark.gpu
 
 MODES = ["clamp", "mirror", "repeat", "constant"]
-VARIANTS = ["auto", "block", "warp", "naive"]
+VARIANTS = ["auto", "tma", "block", "warp", "naive"]
 
 
 @pytest.fixture(scope="module")
