@@ -245,7 +245,8 @@ def run_isp(args):
         for k in range(max(args.warmup, 1)):      # warm-up (also loads every kernel)
             step(k)
     torch.cuda.synchronize()
-    graphs = []
+    graphs = []          # graphs[ph]: one step of rotation phase ph (remainders)
+    graph_cycle = None   # one graph of a full rotation cycle (nphase steps, >= 12 launches)
     if use_graph:
         try:
             for ph in range(nphase):
@@ -253,20 +254,28 @@ def run_isp(args):
                 with torch.cuda.graph(g, stream=stream):
                     step(ph)
                 graphs.append(g)
-            for g in graphs:
+            graph_cycle = torch.cuda.CUDAGraph()
+            with torch.cuda.graph(graph_cycle, stream=stream):
+                for ph in range(nphase):
+                    step(ph)
+            for g in graphs + [graph_cycle]:
                 g.replay()
             torch.cuda.synchronize()
         except Exception as e:  # pragma: no cover
             print(f"[bench] graph capture failed ({e}); eager launches", file=sys.stderr)
-            graphs = []
+            graphs, graph_cycle = [], None
             use_graph = False
 
     def run_steps(K, v=variant):
+        """Exactly K steps: K // nphase replays of the cycle graph + the remaining steps."""
         with torch.cuda.stream(stream):
-            for k in range(K):
-                if use_graph and v == variant:
-                    graphs[k % nphase].replay()
-                else:
+            if use_graph and v == variant:
+                for _ in range(K // nphase):
+                    graph_cycle.replay()
+                for k in range(K % nphase):
+                    graphs[k].replay()
+            else:
+                for k in range(K):
                     step(k, v)
 
     plan = isp.isp_last_plan()
@@ -305,7 +314,7 @@ def run_isp(args):
             "kernel": f"variant {args.variant}: " + ("k_staged<OpSepF32<5,5>> (TMA-staged ISP)" if plan["choice"] == 4 else "k_stencil<OpSepF32<5,5>>"),
             "algorithmic_bytes_per_launch": BYTES_PER_PX * N_SIDE * N_SIDE,
             "duration_us": per_launch_us,
-            "duration_method": "timed region / launches (graph replay, kernels back-to-back)"}
+            "duration_method": "timed region / launches (CUDA-graph replay of a full rotation cycle, kernels back-to-back)"}
 
     # ---- ISP vs naive per mode (same methodology, single-GPU variants) ----
     variants = {}

@@ -94,6 +94,7 @@ int num_sms()
 }
 
 constexpr int kMinRowsPerBlock = 8;
+constexpr int kStreamTileRows = 16;
 
 // blocks_per_sm: resident blocks of the kernel that will run (occupancy API); 0 = 8.
 Plan make_plan(int w, int h, int hx, int hy, int px, int tile_w_req, int tile_h_req, int warp_w_req,
@@ -204,13 +205,13 @@ void model(const Plan &p, int w, int h, int mw, int mh, const isp_model_params &
 int blocks_per_sm(const void *fn, int threads, size_t smem = 0)
 {
     static std::mutex mu;
-    static std::unordered_map<const void *, int> cache[9];
+    static std::unordered_map<const void *, std::pair<size_t, int>> cache[9];
     if (!fn) return 0;
     const int slot = smem ? 0 : std::min(8, threads / 32);
     {
         std::lock_guard<std::mutex> lk(mu);
         auto it = cache[slot].find(fn);
-        if (it != cache[slot].end()) return it->second;
+        if (it != cache[slot].end() && it->second.first == smem) return it->second.second;
     }
     int nb = 0;
     if (smem > 48 * 1024 && cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) !=
@@ -221,7 +222,7 @@ int blocks_per_sm(const void *fn, int threads, size_t smem = 0)
         nb = 0;
     }
     std::lock_guard<std::mutex> lk(mu);
-    cache[slot][fn] = nb;
+    cache[slot][fn] = {smem, nb};
     return nb;
 }
 
@@ -261,7 +262,7 @@ using RunFn = cudaError_t (*)(const Desc &);
 // 128*PX, halo rounded up to 16 B (HXA) and Eq. (2)'s x bounds taken with HXA and the
 // 16-B aligned width w_al, so every Body CTA's bulk copies are in bounds (A21).
 struct StagedGeom {
-    int hxa, w_al, sw, stages;
+    int hxa, w_al, sw, stages, rs;
     size_t smem;
 };
 
@@ -269,14 +270,22 @@ StagedGeom staged_geom(int w, int hx, int hy, int px, int esz, int nin)
 {
     StagedGeom sg{};
     const int tw = STAGED_WARPS * 32 * px;
-    sg.hxa = (int)(ceil_div((long long)hx * esz, 16) * 16 / esz);
+    // halo rounded up to a whole number of 32-B L2 sectors: the bulk copies then start
+    // and end on sector boundaries (16-B-aligned copies straddle sectors)
+    int align = 32;
+    if (const char *e = getenv("ISP_HALO_ALIGN")) align = std::max(16, atoi(e));
+    sg.hxa = (int)(ceil_div((long long)hx * esz, align) * align / esz);
     sg.w_al = (int)(((long long)w * esz / 16) * 16 / esz);
     sg.sw = tw + 2 * sg.hxa;
-    const long long mh = 2 * hy + 1;
-    const long long stage_bytes = mh * nin * sg.sw * esz;
-    sg.stages = (int)std::min<long long>(16, std::max<long long>(3, ceil_div(24 * 1024, stage_bytes)));
-    if (const char *e = getenv("ISP_STAGES")) sg.stages = std::max(2, std::min(16, atoi(e)));
-    sg.smem = 256 + (size_t)sg.stages * stage_bytes;
+    // ring of single-row slots, >= 4 slots / ~8 KB of rows in flight per CTA: measured
+    // best on B200 (knobs ISP_RS, ISP_STAGES)
+    const long long row_bytes = (long long)nin * sg.sw * esz;
+    sg.rs = 1;
+    if (const char *e = getenv("ISP_RS")) sg.rs = std::max(1, std::min(16, atoi(e)));
+    const long long slot_bytes = row_bytes * sg.rs;
+    sg.stages = (int)std::min<long long>(32, std::max<long long>(4, ceil_div(8 * 1024, slot_bytes)));
+    if (const char *e = getenv("ISP_STAGES")) sg.stages = std::max(2, std::min(32, atoi(e)));
+    sg.smem = 512 + (size_t)sg.stages * slot_bytes;
     return sg;
 }
 
@@ -320,7 +329,8 @@ isp_status_t resolve_and_launch(Desc &d, int fam, int w, int h, int mw, int mh, 
     tma_ok = tma_ok && !direct && fn_of(DISP_TMA) != nullptr && g_override_wx == 0;
     const int nb_naive = blocks_per_sm(fn_of(naive_disp), threads);
     const int nb_stream = blocks_per_sm(fn_of(p0.wx > 1 ? DISP_WARP : DISP_BLOCK), threads);
-    const int nb_tma = tma_ok ? blocks_per_sm(fn_of(DISP_TMA), STAGED_THREADS, sg.smem) : 0;
+    int nb_tma = tma_ok ? blocks_per_sm(fn_of(DISP_TMA), STAGED_THREADS, sg.smem) : 0;
+    if (const char *e = getenv("ISP_CTAS_PER_SM")) nb_tma = std::min(nb_tma, std::max(1, atoi(e)));
     if (tma_ok && nb_tma <= 0) tma_ok = false;
 
     isp_variant_t chosen = v;
@@ -332,7 +342,10 @@ isp_status_t resolve_and_launch(Desc &d, int fam, int w, int h, int mw, int mh, 
             apply_staged_bounds(q, w, px, sg);
             return q;
         }
-        return make_plan(w, h, hx, hy, px, 0, 0, 0, rr, c == ISP_NAIVE ? nb_naive : nb_stream);
+        // streaming / naive kernels: uniform tiles of kStreamTileRows rows (Eq. 2 verbatim);
+        // several waves of small blocks hide their load latency best (measured)
+        return make_plan(w, h, hx, hy, px, 0, g_override_ty > 0 ? 0 : kStreamTileRows, 0, rr,
+                         c == ISP_NAIVE ? nb_naive : nb_stream);
     };
     Plan p = plan_for(chosen);
     isp_plan_info info{};
@@ -359,6 +372,7 @@ isp_status_t resolve_and_launch(Desc &d, int fam, int w, int h, int mw, int mh, 
     d.g.w_al = sg.w_al;
     d.g.sw = sg.sw;
     d.g.stages = sg.stages;
+    d.g.rs = sg.rs;
     d.grid = dim3(p.nx, p.ny, 1);
     d.block = dim3(chosen == ISP_TMA ? STAGED_THREADS : threads, 1, 1);
     d.smem = chosen == ISP_TMA ? sg.smem : 0;

@@ -21,7 +21,7 @@ template <int MW_, int MH_>
 struct OpConvF32 {
     using Tin = float;
     static constexpr int NIN = 1, PX = 4, HX = MW_ / 2, HY = MH_ / 2, MH = MH_, SEGW = PX + 2 * HX;
-    static constexpr int PFMAX = 1;
+    static constexpr int PFMAX = 0;
     static constexpr bool ROW_DIRECT = false;
     struct Params {
         Geom g;
@@ -44,12 +44,15 @@ struct OpConvF32 {
 #pragma unroll
         for (int k = 0; k < SEGW; ++k) h.s[k] = seg[0][k];
     }
+    // FIRST: the output row's first tap (j == 0) initialises the accumulator
+    template <bool FIRST>
     __device__ __forceinline__ static void vacc(const Params &p, int j, const H &h, A &a)
     {
 #pragma unroll
         for (int i = 0; i < MW_; ++i)
 #pragma unroll
-            for (int e = 0; e < PX; ++e) a.v[e] = fmaf(p.mask[j * MW_ + i], h.s[e + i], a.v[e]);
+            for (int e = 0; e < PX; ++e)
+                a.v[e] = (FIRST && i == 0) ? p.mask[j * MW_] * h.s[e] : fmaf(p.mask[j * MW_ + i], h.s[e + i], a.v[e]);
     }
     template <int CK>
     __device__ __forceinline__ static void store(const Params &p, const A &a, int x0, int y)
@@ -66,7 +69,7 @@ template <int MW_, int MH_>
 struct OpSepF32 {
     using Tin = float;
     static constexpr int NIN = 1, PX = 4, HX = MW_ / 2, HY = MH_ / 2, MH = MH_, SEGW = PX + 2 * HX;
-    static constexpr int PFMAX = 1;
+    static constexpr int PFMAX = 0;
     static constexpr bool ROW_DIRECT = false;
     struct Params {
         Geom g;
@@ -95,10 +98,11 @@ struct OpSepF32 {
             h.v[e] = t;
         }
     }
+    template <bool FIRST>
     __device__ __forceinline__ static void vacc(const Params &p, int j, const H &h, A &a)
     {
 #pragma unroll
-        for (int e = 0; e < PX; ++e) a.v[e] = fmaf(p.col[j], h.v[e], a.v[e]);
+        for (int e = 0; e < PX; ++e) a.v[e] = FIRST ? p.col[j] * h.v[e] : fmaf(p.col[j], h.v[e], a.v[e]);
     }
     template <int CK>
     __device__ __forceinline__ static void store(const Params &p, const A &a, int x0, int y)
@@ -129,7 +133,7 @@ template <int MW_, int MH_>
 struct OpConvU8 {
     using Tin = uint8_t;
     static constexpr int NIN = 1, PX = 8, HX = MW_ / 2, HY = MH_ / 2, MH = MH_, SEGW = PX + 2 * HX;
-    static constexpr int PFMAX = 1;
+    static constexpr int PFMAX = 0;
     static constexpr bool ROW_DIRECT = false;
     struct Params {
         Geom g;
@@ -153,12 +157,14 @@ struct OpConvU8 {
 #pragma unroll
         for (int k = 0; k < SEGW; ++k) h.s[k] = seg[0][k];
     }
+    template <bool FIRST>
     __device__ __forceinline__ static void vacc(const Params &p, int j, const H &h, A &a)
     {
 #pragma unroll
         for (int i = 0; i < MW_; ++i)
 #pragma unroll
-            for (int e = 0; e < PX; ++e) a.v[0][e] += p.mask[j * MW_ + i] * h.s[e + i];
+            for (int e = 0; e < PX; ++e)
+                a.v[0][e] = ((FIRST && i == 0) ? 0 : a.v[0][e]) + p.mask[j * MW_ + i] * h.s[e + i];
     }
     template <int CK>
     __device__ __forceinline__ static void store(const Params &p, const A &a, int x0, int y)
@@ -175,7 +181,7 @@ template <int MW_, int MH_>
 struct OpSepU8 {
     using Tin = uint8_t;
     static constexpr int NIN = 1, PX = 8, HX = MW_ / 2, HY = MH_ / 2, MH = MH_, SEGW = PX + 2 * HX;
-    static constexpr int PFMAX = 1;
+    static constexpr int PFMAX = 0;
     static constexpr bool ROW_DIRECT = false;
     struct Params {
         Geom g;
@@ -205,10 +211,11 @@ struct OpSepU8 {
             h.v[e] = t;
         }
     }
+    template <bool FIRST>
     __device__ __forceinline__ static void vacc(const Params &p, int j, const H &h, A &a)
     {
 #pragma unroll
-        for (int e = 0; e < PX; ++e) a.v[0][e] += p.col[j] * h.v[e];
+        for (int e = 0; e < PX; ++e) a.v[0][e] = (FIRST ? 0 : a.v[0][e]) + p.col[j] * h.v[e];
     }
     template <int CK>
     __device__ __forceinline__ static void store(const Params &p, const A &a, int x0, int y)
@@ -238,7 +245,7 @@ __device__ __forceinline__ int isqrt_round(int n)
 struct OpSobel {
     using Tin = uint8_t;
     static constexpr int NIN = 1, PX = 8, HX = 1, HY = 1, MH = 3, SEGW = PX + 2;
-    static constexpr int PFMAX = 1;
+    static constexpr int PFMAX = 0;
     static constexpr bool ROW_DIRECT = false;
     struct Params {
         Geom g;
@@ -265,12 +272,14 @@ struct OpSobel {
             h.df[e] = c - a;
         }
     }
+    template <bool FIRST>
     __device__ __forceinline__ static void vacc(const Params &, int j, const H &h, A &a)
     {
 #pragma unroll
         for (int e = 0; e < PX; ++e) {
-            a.v[0][e] += (j == 1 ? 2 : 1) * h.df[e];
-            if (j != 1) a.v[1][e] += (j - 1) * h.sm[e];
+            a.v[0][e] = (FIRST ? 0 : a.v[0][e]) + (j == 1 ? 2 : 1) * h.df[e];
+            if (FIRST) a.v[1][e] = (j - 1) * h.sm[e];
+            else if (j != 1) a.v[1][e] += (j - 1) * h.sm[e];
         }
     }
     template <int CK>
@@ -303,7 +312,7 @@ struct OpSobel {
 struct OpLaplace5 {
     using Tin = uint8_t;
     static constexpr int NIN = 1, PX = 8, HX = 2, HY = 2, MH = 5, SEGW = PX + 4;
-    static constexpr int PFMAX = 1;
+    static constexpr int PFMAX = 0;
     static constexpr bool ROW_DIRECT = false;
     struct Params {
         Geom g;
@@ -331,11 +340,12 @@ struct OpLaplace5 {
             h.ctr[e] = seg[0][e + 2];
         }
     }
+    template <bool FIRST>
     __device__ __forceinline__ static void vacc(const Params &, int j, const H &h, A &a)
     {
 #pragma unroll
         for (int e = 0; e < PX; ++e) {
-            a.v[0][e] += h.box[e];
+            a.v[0][e] = (FIRST ? 0 : a.v[0][e]) + h.box[e];
             if (j == 2) a.v[1][e] = h.ctr[e];
         }
     }
@@ -354,7 +364,7 @@ struct OpLaplace5 {
 struct OpHarris {
     using Tin = int16_t;
     static constexpr int NIN = 2, PX = 4, HX = 1, HY = 1, MH = 3, SEGW = PX + 2;
-    static constexpr int PFMAX = 1;
+    static constexpr int PFMAX = 0;
     static constexpr bool ROW_DIRECT = false;
     struct Params {
         Geom g;
@@ -389,14 +399,15 @@ struct OpHarris {
             h.xy[e] = pxy[e] + 2 * pxy[e + 1] + pxy[e + 2];
         }
     }
+    template <bool FIRST>
     __device__ __forceinline__ static void vacc(const Params &, int j, const H &h, A &a)
     {
         const int wj = (j == 1) ? 2 : 1;
 #pragma unroll
         for (int e = 0; e < PX; ++e) {
-            a.v[0][e] += wj * h.xx[e];
-            a.v[1][e] += wj * h.yy[e];
-            a.v[2][e] += wj * h.xy[e];
+            a.v[0][e] = (FIRST ? 0 : a.v[0][e]) + wj * h.xx[e];
+            a.v[1][e] = (FIRST ? 0 : a.v[1][e]) + wj * h.yy[e];
+            a.v[2][e] = (FIRST ? 0 : a.v[2][e]) + wj * h.xy[e];
         }
     }
     template <int CK>
@@ -449,6 +460,7 @@ struct OpAtrous {
 #pragma unroll
         for (int e = 0; e < PX; ++e) h.v[e] = fmaf(0.25f, seg[0][e + 2 * D], fmaf(0.5f, seg[0][e + D], 0.25f * seg[0][e]));
     }
+    template <bool FIRST>
     __device__ __forceinline__ static void vacc(const Params &, int j, const H &h, A &a)
     {
         const float wj = (j == D) ? 0.5f : 0.25f;

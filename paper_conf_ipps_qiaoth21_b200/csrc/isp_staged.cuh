@@ -20,7 +20,8 @@ namespace ispk {
 
 constexpr int kStagedComputeWarps = 4;
 constexpr int kStagedThreads = 32 * (kStagedComputeWarps + 1);
-constexpr int kStagedBarrierBytes = 256;  // full[16] + empty[16] mbarriers
+constexpr int kStagedMaxStages = 32;
+constexpr int kStagedBarrierBytes = 512;  // full[32] + empty[32] mbarriers
 
 __device__ __forceinline__ uint32_t smem_u32(const void *p) { return (uint32_t)__cvta_generic_to_shared(p); }
 
@@ -56,6 +57,32 @@ __device__ __forceinline__ void bulk_g2s(void *dst, const void *src, uint32_t by
                  : "memory");
 }
 __device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
+// 4-byte async copy global -> shared (LDGSTS) and an mbarrier arrive that fires when
+// all of this thread's prior cp.async copies have landed (count not incremented).
+__device__ __forceinline__ void cp_async4(void *dst, const void *src)
+{
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_async_mbar_arrive_noinc(uint64_t *b)
+{
+    asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(smem_u32(b)) : "memory");
+}
+
+// Global column the fix-up of column x reads (x outside the bulk-copied range), or -1
+// when no stored output reads it (beyond the window's reach: left as is).
+template <class Op, int MODE, int CK>
+__device__ __forceinline__ int fixup_source(int x, const Geom &g)
+{
+    if (x >= 0 && x < g.w) return x;
+    if (x < -Op::HX || x >= g.w + Op::HX) return -1;
+    if constexpr ((CK & CK_L) != 0) {
+        if (x < 0) return bmap<MODE, true, false, false>(x, g.w);
+    }
+    if constexpr ((CK & CK_R) != 0) {
+        if (x >= g.w) return bmap<MODE, false, true, false>(x, g.w);
+    }
+    return -1;
+}
 __device__ __forceinline__ void fence_mbar_init() { asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory"); }
 
 template <int N>
@@ -128,20 +155,23 @@ __device__ __forceinline__ void staged_body(const typename Op::Params &p, unsign
     const Geom &g = p.g;
     const int S = g.stages, SW = g.sw, HXA = g.hxa;
     uint64_t *full = reinterpret_cast<uint64_t *>(smem);
-    uint64_t *empty = full + 16;
+    uint64_t *empty = full + kStagedMaxStages;
     T *buf = reinterpret_cast<T *>(smem + kStagedBarrierBytes);
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     int y0, rows;
     block_rows(g, blockIdx.y, gridDim.y, y0, rows);
-    const int nr = rows + 2 * HY;
-    const int nfill = (nr + MH - 1) / MH;
+    const int nr = rows + 2 * HY;            // input rows of this CTA (one ring slot each)
     const int X0 = blockIdx.x * TW;          // first output column of the CTA
     const int XS = X0 - HXA;                 // global column of smem column 0
-    const size_t stage_elems = (size_t)MH * NIN * SW;
+    const int RS = g.rs;                     // rows per ring slot
+    const size_t row_elems = (size_t)NIN * SW, slot_elems = (size_t)RS * row_elems;
 
+    // L/R CTAs of 4-byte types fetch their fix-up columns with cp.async: every producer
+    // lane then arrives on the full barrier when its copies land (32 extra arrivals)
+    constexpr bool ASYNC_FIX = (CK & (CK_L | CK_R)) != 0 && sizeof(T) == 4 && MODE != CONSTANT;
     if (threadIdx.x == 0) {
         for (int s = 0; s < S; ++s) {
-            mbar_init(&full[s], 1);
+            mbar_init(&full[s], ASYNC_FIX ? 33 : 1);
             mbar_init(&empty[s], NWC);
         }
         fence_mbar_init();
@@ -149,70 +179,71 @@ __device__ __forceinline__ void staged_body(const typename Op::Params &p, unsign
     __syncthreads();
 
     if (warp == NWC) {
-        // ---------------- producer warp ----------------
-        for (int i = 0; i < nfill; ++i) {
-            const int s = i % S;
-            if (i >= S) mbar_wait(&empty[s], ((i / S) - 1) & 1);
-            T *sb = buf + (size_t)s * stage_elems;
-            int yyk[MH], csk[MH], cek[MH];
-            bool okk[MH];
+        // ---------------- producer warp: RS input rows per ring slot ----------------
+        int s = 0, nfill = 0;
+        uint32_t ph = 0;
+        for (int f0 = 0; f0 < nr; f0 += RS, ++nfill) {
+            if (nfill >= S) mbar_wait(&empty[s], ph ^ 1);
+            const int nrow = min(RS, nr - f0);
+            T *sb = buf + (size_t)s * slot_elems;
             uint32_t bytes = 0;
-#pragma unroll
-            for (int k = 0; k < MH; ++k) {
-                const int r = i * MH + k;
-                bool rowok = false;
-                int yy = 0, cs = 0, ce = 0;
-                if (r < nr) {
-                    yy = map_row<MODE, CK>(y0 - HY + r, g, rowok);
-                    cs = XS;
-                    ce = X0 + TW + HXA;
-                    if constexpr ((CK & CK_L) != 0) cs = max(cs, 0);
-                    if constexpr ((CK & CK_R) != 0) ce = min(ce, g.w_al);
-                    if (MODE == CONSTANT && !rowok) ce = cs;  // whole row = C
-                    if (ce > cs) bytes += (uint32_t)(ce - cs) * (uint32_t)sizeof(T) * NIN;
-                }
-                yyk[k] = yy;
-                okk[k] = (r < nr) && (MODE != CONSTANT || rowok);
-                csk[k] = cs;
-                cek[k] = ce;
+            for (int k = 0; k < nrow; ++k) {
+                bool rowok;
+                map_row<MODE, CK>(y0 - HY + f0 + k, g, rowok);
+                int cs = XS, ce = X0 + TW + HXA;
+                if constexpr ((CK & CK_L) != 0) cs = max(cs, 0);
+                if constexpr ((CK & CK_R) != 0) ce = min(ce, g.w_al);
+                if (!(MODE == CONSTANT && !rowok) && ce > cs) bytes += (uint32_t)(ce - cs) * (uint32_t)sizeof(T) * NIN;
             }
-            if (lane == 0) {
-                mbar_expect_tx(&full[s], bytes);
+            if (lane == 0) mbar_expect_tx(&full[s], bytes);
+            for (int k = 0; k < nrow; ++k) {
+                bool rowok;
+                const int yy = map_row<MODE, CK>(y0 - HY + f0 + k, g, rowok);
+                int cs = XS, ce = X0 + TW + HXA;
+                if constexpr ((CK & CK_L) != 0) cs = max(cs, 0);
+                if constexpr ((CK & CK_R) != 0) ce = min(ce, g.w_al);
+                if (MODE == CONSTANT && !rowok) ce = cs;  // whole row = C
+                T *rb = sb + (size_t)k * row_elems;
+                if (lane == 0 && ce > cs)
 #pragma unroll
-                for (int k = 0; k < MH; ++k)
-                    if (cek[k] > csk[k])
-#pragma unroll
-                        for (int c = 0; c < NIN; ++c)
-                            bulk_g2s(sb + ((size_t)k * NIN + c) * SW + (csk[k] - XS),
-                                     p.in[c] + (ptrdiff_t)yyk[k] * g.in_pitch + csk[k],
-                                     (uint32_t)(cek[k] - csk[k]) * (uint32_t)sizeof(T), &full[s]);
-            }
-            if constexpr (CK != 0) {
-                // border fix-ups (this region's sides only): generic stores by the warp
-#pragma unroll
-                for (int k = 0; k < MH; ++k) {
-                    const int r = i * MH + k;
-                    if (r >= nr) continue;
+                    for (int c = 0; c < NIN; ++c)
+                        bulk_g2s(rb + (size_t)c * SW + (cs - XS), p.in[c] + (ptrdiff_t)yy * g.in_pitch + cs,
+                                 (uint32_t)(ce - cs) * (uint32_t)sizeof(T), &full[s]);
+                if constexpr (CK != 0) {
+                    // border fix-ups, this region's sides only (<= HXA columns per row):
+                    // cp.async of the pattern's source column (4-byte types), else a
+                    // synchronous copy; Constant: the constant
 #pragma unroll
                     for (int c = 0; c < NIN; ++c) {
-                        T *dst = sb + ((size_t)k * NIN + c) * SW;
-                        if (MODE == CONSTANT && !okk[k]) {
+                        T *dst = rb + (size_t)c * SW;
+                        if (MODE == CONSTANT && !rowok) {
                             for (int x = lane; x < SW; x += 32) dst[x] = p.cval;
                             continue;
                         }
-                        const T *src = p.in[c] + (ptrdiff_t)yyk[k] * g.in_pitch;
+                        const T *src = p.in[c] + (ptrdiff_t)yy * g.in_pitch;
+                        auto fix = [&](int x) {
+                            if constexpr (MODE == CONSTANT) {
+                                dst[x - XS] = (x >= 0 && x < g.w) ? __ldg(src + x) : p.cval;
+                            } else {
+                                const int xs = fixup_source<Op, MODE, CK>(x, g);
+                                if (xs < 0) return;
+                                if constexpr (ASYNC_FIX) cp_async4(dst + (x - XS), src + xs);
+                                else dst[x - XS] = __ldg(src + xs);
+                            }
+                        };
                         if constexpr ((CK & CK_L) != 0)
-                            for (int x = XS + lane; x < csk[k]; x += 32)
-                                dst[x - XS] = fixup_value<Op, MODE, CK>(src, x, g, p.cval);
+                            for (int x = XS + lane; x < cs; x += 32) fix(x);
                         if constexpr ((CK & CK_R) != 0)
-                            for (int x = cek[k] + lane; x < X0 + TW + HXA; x += 32)
-                                dst[x - XS] = fixup_value<Op, MODE, CK>(src, x, g, p.cval);
+                            for (int x = ce + lane; x < X0 + TW + HXA; x += 32) fix(x);
                     }
                 }
-                fence_proxy_async();  // order generic writes before later async writes
             }
+            if constexpr (ASYNC_FIX) cp_async_mbar_arrive_noinc(&full[s]);
+            if constexpr (MODE == CONSTANT && (CK & (CK_T | CK_B)) != 0)
+                fence_proxy_async();  // generic row fills before later bulk (async-proxy) writes
             __syncwarp();
             if (lane == 0) mbar_arrive(&full[s]);
+            if (++s == S) { s = 0; ph ^= 1; }
         }
         return;
     }
@@ -223,41 +254,46 @@ __device__ __forceinline__ void staged_body(const typename Op::Params &p, unsign
     typename Op::A acc[MH];
 #pragma unroll
     for (int k = 0; k < MH; ++k) Op::zero(acc[k]);
-    for (int i = 0; i < nfill; ++i) {
-        const int s = i % S;
-        mbar_wait(&full[s], (i / S) & 1);
-        const T *sb = buf + (size_t)s * stage_elems;
-        if (g.dbg == 1) {
-            __syncwarp();
-            if (lane == 0) mbar_arrive(&empty[s]);
-            continue;
-        }
+    int s = 0, kr = 0;
+    uint32_t ph = 0;
+    for (int r0 = 0; r0 < nr; r0 += MH) {
 #pragma unroll
         for (int k = 0; k < MH; ++k) {
-            const int r = i * MH + k;
+            const int r = r0 + k;
             if (r < nr) {
-                const T *srow[NIN];
-#pragma unroll
-                for (int c = 0; c < NIN; ++c) srow[c] = sb + ((size_t)k * NIN + c) * SW + HXA + xoff;
+                if (kr == 0) mbar_wait(&full[s], ph);
+                const T *rb = buf + (size_t)s * slot_elems + (size_t)kr * row_elems;
                 RawRow<Op> rr;
-                load_row_smem<Op>(srow, rr);
+                if (g.dbg != 1) {
+                    const T *srow[NIN];
+#pragma unroll
+                    for (int c = 0; c < NIN; ++c) srow[c] = rb + (size_t)c * SW + HXA + xoff;
+                    load_row_smem<Op>(srow, rr);
+                }
+                if (++kr == RS || r == nr - 1) {
+                    __syncwarp();
+                    if (lane == 0) mbar_arrive(&empty[s]);  // release: the slot's rows are in registers
+                    kr = 0;
+                    if (++s == S) { s = 0; ph ^= 1; }
+                }
+                if (g.dbg == 1) continue;
                 T seg[NIN][SEGW];
                 unpack_row<Op>(rr, seg);
                 typename Op::H hs;
                 Op::hrow(p, seg, hs);
+                // every tap unconditionally: j == 0 initialises the row's accumulator, so
+                // rows before the strip (o < 0) or past it (o >= rows) only touch slots
+                // that are re-initialised before use or never stored
+                Op::template vacc<true>(p, 0, hs, acc[k]);
 #pragma unroll
-                for (int j = 0; j < MH; ++j) {
+                for (int j = 1; j < MH; ++j) {
                     if (!Op::row_used(j)) continue;
-                    const int o = r - j;
-                    if (o >= 0 && o < rows) Op::vacc(p, j, hs, acc[(k - j + MH) % MH]);
+                    Op::template vacc<false>(p, j, hs, acc[(k - j + MH) % MH]);
                 }
                 const int o = r - (MH - 1);
                 if (o >= 0 && g.dbg != 2) Op::template store<CK & CK_R>(p, acc[(k + 1) % MH], x0, y0 + o);
-                Op::zero(acc[(k + 1) % MH]);
             }
         }
-        __syncwarp();
-        if (lane == 0) mbar_arrive(&empty[s]);
     }
 }
 

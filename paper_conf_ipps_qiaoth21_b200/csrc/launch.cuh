@@ -1,7 +1,7 @@
 // launch.cuh -- template glue: pick the (op, mode, dispatch) kernel instance and launch it.
 #pragma once
 #include <mutex>
-#include <unordered_set>
+#include <unordered_map>
 
 #include "isp_direct.cuh"
 #include "isp_ops.cuh"
@@ -55,12 +55,13 @@ cudaError_t launch_params(const void *fn, const Desc &d, const P &p)
     if (!fn) return cudaErrorNotSupported;
     if (d.smem > 48 * 1024) {
         static std::mutex mu;
-        static std::unordered_set<const void *> done;
+        static std::unordered_map<const void *, size_t> done;
         std::lock_guard<std::mutex> lk(mu);
-        if (!done.count(fn)) {
+        auto it = done.find(fn);
+        if (it == done.end() || it->second < d.smem) {
             cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)d.smem);
             if (e != cudaSuccess) return e;
-            done.insert(fn);
+            done[fn] = d.smem;
         }
     }
     void *args[] = {const_cast<P *>(&p)};
