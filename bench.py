@@ -62,10 +62,14 @@ def peaks():
 
 
 def ncu_traffic():
-    """Per-launch DRAM bytes of the dominant kernel from the committed ncu --set full summary."""
-    p = os.path.join(ROOT, "profiles", "ncu_summary.json")
+    """Per-launch DRAM bytes (read + write) of the dominant kernel from the newest committed
+    `ncu --set full` summary (profiles/r<NN>_ncu_summary.json, tools/ncu_summary.py)."""
+    import glob
+    paths = sorted(glob.glob(os.path.join(ROOT, "profiles", "r*_ncu_summary.json")))
+    if not paths:
+        return None
     try:
-        d = json.load(open(p))
+        d = json.load(open(paths[-1]))
         return d.get("dominant_kernel", {}).get("dram_bytes_per_launch")
     except Exception:
         return None

@@ -209,6 +209,12 @@ isp_status_t isp_shard_filter_u8(isp_shard_ctx *ctx, uint8_t *strip, int w, int 
                                  const int32_t *mask, int mw, int mh, int32_t divisor, int border_mode,
                                  int const_val, uint8_t *out, int out_pitch, isp_variant_t variant,
                                  isp_stream_t stream, isp_stream_t comm_stream);
+/* The launch part of isp_shard_filter_f32 for rank `rank` of `nranks`, without any
+ * communication: the caller has already filled the strip's halo rows (e.g. its own
+ * exchange, or a single-GPU emulation of the strips in tests). */
+isp_status_t isp_shard_filter_local_f32(float *strip, int w, int H, int pitch, int halo, int rank, int nranks,
+                                        const float *mask, int mw, int mh, int border_mode, float const_val,
+                                        float *out, int out_pitch, isp_variant_t variant, isp_stream_t stream);
 isp_status_t isp_shard_destroy(isp_shard_ctx *ctx);
 
 /* Tuning: force the launch shape (warps per block along x, tile height in rows);

@@ -26,7 +26,7 @@ __all__ = [
     "isp_sobel_u8", "isp_laplace5_u8", "isp_harris_u8", "isp_bilateral_f32", "isp_atrous_f32",
     "isp_night_f32", "isp_plan", "isp_model_defaults", "isp_last_plan", "isp_set_launch_override",
     "isp_shard_unique_id", "isp_shard_init", "isp_shard_rows", "isp_shard_schedule",
-    "isp_shard_filter_f32", "isp_shard_filter_u8", "isp_shard_destroy",
+    "isp_shard_filter_f32", "isp_shard_filter_u8", "isp_shard_filter_local_f32", "isp_shard_destroy",
 ]
 
 CLAMP, MIRROR, REPEAT, CONSTANT = 0, 1, 2, 3
@@ -109,6 +109,7 @@ _SIGS = {
     "isp_shard_filter_f32": [_P, _P, _I, _I, _I, _I, _P, _I, _I, _I, _F, _P, _I, _I, _P, _P],
     "isp_shard_filter_u8": [_P, _P, _I, _I, _I, _I, _P, _I, _I, ctypes.c_int32, _I, _I, _P, _I, _I, _P, _P],
     "isp_shard_destroy": [_P],
+    "isp_shard_filter_local_f32": [_P, _I, _I, _I, _I, _I, _I, _P, _I, _I, _I, _F, _P, _I, _I, _P],
 }
 
 _lib = None
@@ -379,6 +380,21 @@ def isp_shard_filter_u8(ctx, strip, H, halo, mask, divisor, border_mode, const_v
     _check(lib().isp_shard_filter_u8(ctx, strip.data_ptr(), w, int(H), pitch, int(halo), mp, mw, mh, int(divisor),
                                      _mode(border_mode), int(const_val), out.data_ptr(), out.shape[1],
                                      _variant(variant), _stream(strip, stream), ctypes.c_void_p(cs.cuda_stream)))
+    return out
+
+
+def isp_shard_filter_local_f32(strip, H, halo, rank, nranks, mask, border_mode, const_val=0.0, out=None,
+                               variant=AUTO, w=None, stream=None):
+    """Strip launches of one rank without communication (halo rows already filled)."""
+    _img(strip, torch.float32, "strip")
+    w, _, pitch = _geom(strip, w)
+    m, mp = _host(mask, ctypes.c_float)
+    mh, mw = m.shape
+    if out is None:
+        out = torch.empty((strip.shape[0] - 2 * halo, w), dtype=torch.float32, device=strip.device)
+    _check(lib().isp_shard_filter_local_f32(strip.data_ptr(), w, int(H), pitch, int(halo), int(rank), int(nranks), mp,
+                                            mw, mh, _mode(border_mode), float(const_val), out.data_ptr(),
+                                            out.shape[1], _variant(variant), _stream(strip, stream)))
     return out
 
 

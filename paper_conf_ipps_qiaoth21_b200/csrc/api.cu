@@ -386,6 +386,7 @@ isp_status_t resolve_and_launch(Desc &d, int fam, int w, int h, int mw, int mh, 
     d.disp = chosen == ISP_TMA ? DISP_TMA : chosen == ISP_WARP ? DISP_WARP : chosen == ISP_BLOCK ? DISP_BLOCK
                                                                                                : naive_disp;
     d.g.warp_level = chosen == ISP_WARP;
+    d.g.mode = d.mode;
     if (const char *e = getenv("ISP_DEBUG_STAGED")) d.g.dbg = atoi(e);
     g_last_plan = info;
     cudaError_t e = run(d);

@@ -10,6 +10,26 @@
 namespace ispk {
 
 template <int PX> struct AccF { float v[PX]; };
+
+// Packed FP32 FMA (sm_100 FFMA2): (a0, a1) = fma(c, (b0, b1), (a0, a1)) -- two IEEE fmaf
+// per instruction, bitwise identical to the scalar form; c is broadcast.
+__device__ __forceinline__ void fma2(float &a0, float &a1, float c, float b0, float b1)
+{
+    unsigned long long aa, bb, cc;
+    asm("mov.b64 %0, {%1, %2};" : "=l"(aa) : "f"(a0), "f"(a1));
+    asm("mov.b64 %0, {%1, %2};" : "=l"(bb) : "f"(b0), "f"(b1));
+    asm("mov.b64 %0, {%1, %1};" : "=l"(cc) : "f"(c));
+    asm("fma.rn.f32x2 %0, %1, %2, %0;" : "+l"(aa) : "l"(cc), "l"(bb));
+    asm("mov.b64 {%0, %1}, %2;" : "=f"(a0), "=f"(a1) : "l"(aa));
+}
+__device__ __forceinline__ void mul2(float &a0, float &a1, float c, float b0, float b1)
+{
+    unsigned long long aa, bb, cc;
+    asm("mov.b64 %0, {%1, %2};" : "=l"(bb) : "f"(b0), "f"(b1));
+    asm("mov.b64 %0, {%1, %1};" : "=l"(cc) : "f"(c));
+    asm("mul.rn.f32x2 %0, %1, %2;" : "=l"(aa) : "l"(cc), "l"(bb));
+    asm("mov.b64 {%0, %1}, %2;" : "=f"(a0), "=f"(a1) : "l"(aa));
+}
 template <int PX, int NC> struct AccI { int v[NC][PX]; };
 
 // ---------------------------------------------------------------------------------
@@ -48,6 +68,7 @@ struct OpConvF32 {
     template <bool FIRST>
     __device__ __forceinline__ static void vacc(const Params &p, int j, const H &h, A &a)
     {
+        // scalar FFMA: the packed form (fma2) makes ptxas take ~20 min on the 7x7 instance
 #pragma unroll
         for (int i = 0; i < MW_; ++i)
 #pragma unroll
@@ -91,18 +112,23 @@ struct OpSepF32 {
     __device__ __forceinline__ static void hrow(const Params &p, const float (&seg)[1][SEGW], H &h)
     {
 #pragma unroll
-        for (int e = 0; e < PX; ++e) {
-            float t = p.row[0] * seg[0][e];
+        for (int e = 0; e < PX; e += 2) {
+            float t0, t1;
+            mul2(t0, t1, p.row[0], seg[0][e], seg[0][e + 1]);
 #pragma unroll
-            for (int i = 1; i < MW_; ++i) t = fmaf(p.row[i], seg[0][e + i], t);
-            h.v[e] = t;
+            for (int i = 1; i < MW_; ++i) fma2(t0, t1, p.row[i], seg[0][e + i], seg[0][e + i + 1]);
+            h.v[e] = t0;
+            h.v[e + 1] = t1;
         }
     }
     template <bool FIRST>
     __device__ __forceinline__ static void vacc(const Params &p, int j, const H &h, A &a)
     {
 #pragma unroll
-        for (int e = 0; e < PX; ++e) a.v[e] = FIRST ? p.col[j] * h.v[e] : fmaf(p.col[j], h.v[e], a.v[e]);
+        for (int e = 0; e < PX; e += 2) {
+            if (FIRST) mul2(a.v[e], a.v[e + 1], p.col[j], h.v[e], h.v[e + 1]);
+            else fma2(a.v[e], a.v[e + 1], p.col[j], h.v[e], h.v[e + 1]);
+        }
     }
     template <int CK>
     __device__ __forceinline__ static void store(const Params &p, const A &a, int x0, int y)

@@ -146,7 +146,89 @@ __device__ __forceinline__ typename Op::Tin fixup_value(const typename Op::Tin *
     }
 }
 
+// Producer warp of a staged CTA (the only mode-dependent code: row maps, fix-ups).
 template <class Op, int MODE, int CK>
+__device__ __forceinline__ void staged_producer(const typename Op::Params &p, uint64_t *full, uint64_t *empty,
+                                                typename Op::Tin *buf, int y0, int nr, int X0)
+{
+    using T = typename Op::Tin;
+    constexpr int HY = Op::HY, PX = Op::PX, NIN = Op::NIN;
+    constexpr int TW = kStagedComputeWarps * 32 * PX;
+    constexpr bool ASYNC_FIX = (CK & (CK_L | CK_R)) != 0 && sizeof(T) == 4 && MODE != CONSTANT;
+    const Geom &g = p.g;
+    const int S = g.stages, SW = g.sw, HXA = g.hxa, RS = g.rs;
+    const int lane = threadIdx.x & 31;
+    const int XS = X0 - HXA;
+    const size_t row_elems = (size_t)NIN * SW, slot_elems = (size_t)RS * row_elems;
+    // ---------------- producer warp: RS input rows per ring slot ----------------
+    int s = 0, nfill = 0;
+    uint32_t ph = 0;
+    for (int f0 = 0; f0 < nr; f0 += RS, ++nfill) {
+        if (nfill >= S) mbar_wait(&empty[s], ph ^ 1);
+        const int nrow = min(RS, nr - f0);
+        T *sb = buf + (size_t)s * slot_elems;
+        uint32_t bytes = 0;
+        for (int k = 0; k < nrow; ++k) {
+            bool rowok;
+            map_row<MODE, CK>(y0 - HY + f0 + k, g, rowok);
+            int cs = XS, ce = X0 + TW + HXA;
+            if constexpr ((CK & CK_L) != 0) cs = max(cs, 0);
+            if constexpr ((CK & CK_R) != 0) ce = min(ce, g.w_al);
+            if (!(MODE == CONSTANT && !rowok) && ce > cs) bytes += (uint32_t)(ce - cs) * (uint32_t)sizeof(T) * NIN;
+        }
+        if (lane == 0) mbar_expect_tx(&full[s], bytes);
+        for (int k = 0; k < nrow; ++k) {
+            bool rowok;
+            const int yy = map_row<MODE, CK>(y0 - HY + f0 + k, g, rowok);
+            int cs = XS, ce = X0 + TW + HXA;
+            if constexpr ((CK & CK_L) != 0) cs = max(cs, 0);
+            if constexpr ((CK & CK_R) != 0) ce = min(ce, g.w_al);
+            if (MODE == CONSTANT && !rowok) ce = cs;  // whole row = C
+            T *rb = sb + (size_t)k * row_elems;
+            if (lane == 0 && ce > cs)
+#pragma unroll
+                for (int c = 0; c < NIN; ++c)
+                    bulk_g2s(rb + (size_t)c * SW + (cs - XS), p.in[c] + (ptrdiff_t)yy * g.in_pitch + cs,
+                             (uint32_t)(ce - cs) * (uint32_t)sizeof(T), &full[s]);
+            if constexpr (CK != 0) {
+                // border fix-ups, this region's sides only (<= HXA columns per row):
+                // cp.async of the pattern's source column (4-byte types), else a
+                // synchronous copy; Constant: the constant
+#pragma unroll
+                for (int c = 0; c < NIN; ++c) {
+                    T *dst = rb + (size_t)c * SW;
+                    if (MODE == CONSTANT && !rowok) {
+                        for (int x = lane; x < SW; x += 32) dst[x] = p.cval;
+                        continue;
+                    }
+                    const T *src = p.in[c] + (ptrdiff_t)yy * g.in_pitch;
+                    auto fix = [&](int x) {
+                        if constexpr (MODE == CONSTANT) {
+                            dst[x - XS] = (x >= 0 && x < g.w) ? __ldg(src + x) : p.cval;
+                        } else {
+                            const int xs = fixup_source<Op, MODE, CK>(x, g);
+                            if (xs < 0) return;
+                            if constexpr (ASYNC_FIX) cp_async4(dst + (x - XS), src + xs);
+                            else dst[x - XS] = __ldg(src + xs);
+                        }
+                    };
+                    if constexpr ((CK & CK_L) != 0)
+                        for (int x = XS + lane; x < cs; x += 32) fix(x);
+                    if constexpr ((CK & CK_R) != 0)
+                        for (int x = ce + lane; x < X0 + TW + HXA; x += 32) fix(x);
+                }
+            }
+        }
+        if constexpr (ASYNC_FIX) cp_async_mbar_arrive_noinc(&full[s]);
+        if constexpr (MODE == CONSTANT && (CK & (CK_T | CK_B)) != 0)
+            fence_proxy_async();  // generic row fills before later bulk (async-proxy) writes
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&full[s]);
+        if (++s == S) { s = 0; ph ^= 1; }
+    }
+}
+
+template <class Op, int CK>
 __device__ __forceinline__ void staged_body(const typename Op::Params &p, unsigned char *smem)
 {
     using T = typename Op::Tin;
@@ -168,10 +250,10 @@ __device__ __forceinline__ void staged_body(const typename Op::Params &p, unsign
 
     // L/R CTAs of 4-byte types fetch their fix-up columns with cp.async: every producer
     // lane then arrives on the full barrier when its copies land (32 extra arrivals)
-    constexpr bool ASYNC_FIX = (CK & (CK_L | CK_R)) != 0 && sizeof(T) == 4 && MODE != CONSTANT;
+    const bool async_fix = (CK & (CK_L | CK_R)) != 0 && sizeof(T) == 4 && g.mode != CONSTANT;
     if (threadIdx.x == 0) {
         for (int s = 0; s < S; ++s) {
-            mbar_init(&full[s], ASYNC_FIX ? 33 : 1);
+            mbar_init(&full[s], async_fix ? 33 : 1);
             mbar_init(&empty[s], NWC);
         }
         fence_mbar_init();
@@ -179,71 +261,11 @@ __device__ __forceinline__ void staged_body(const typename Op::Params &p, unsign
     __syncthreads();
 
     if (warp == NWC) {
-        // ---------------- producer warp: RS input rows per ring slot ----------------
-        int s = 0, nfill = 0;
-        uint32_t ph = 0;
-        for (int f0 = 0; f0 < nr; f0 += RS, ++nfill) {
-            if (nfill >= S) mbar_wait(&empty[s], ph ^ 1);
-            const int nrow = min(RS, nr - f0);
-            T *sb = buf + (size_t)s * slot_elems;
-            uint32_t bytes = 0;
-            for (int k = 0; k < nrow; ++k) {
-                bool rowok;
-                map_row<MODE, CK>(y0 - HY + f0 + k, g, rowok);
-                int cs = XS, ce = X0 + TW + HXA;
-                if constexpr ((CK & CK_L) != 0) cs = max(cs, 0);
-                if constexpr ((CK & CK_R) != 0) ce = min(ce, g.w_al);
-                if (!(MODE == CONSTANT && !rowok) && ce > cs) bytes += (uint32_t)(ce - cs) * (uint32_t)sizeof(T) * NIN;
-            }
-            if (lane == 0) mbar_expect_tx(&full[s], bytes);
-            for (int k = 0; k < nrow; ++k) {
-                bool rowok;
-                const int yy = map_row<MODE, CK>(y0 - HY + f0 + k, g, rowok);
-                int cs = XS, ce = X0 + TW + HXA;
-                if constexpr ((CK & CK_L) != 0) cs = max(cs, 0);
-                if constexpr ((CK & CK_R) != 0) ce = min(ce, g.w_al);
-                if (MODE == CONSTANT && !rowok) ce = cs;  // whole row = C
-                T *rb = sb + (size_t)k * row_elems;
-                if (lane == 0 && ce > cs)
-#pragma unroll
-                    for (int c = 0; c < NIN; ++c)
-                        bulk_g2s(rb + (size_t)c * SW + (cs - XS), p.in[c] + (ptrdiff_t)yy * g.in_pitch + cs,
-                                 (uint32_t)(ce - cs) * (uint32_t)sizeof(T), &full[s]);
-                if constexpr (CK != 0) {
-                    // border fix-ups, this region's sides only (<= HXA columns per row):
-                    // cp.async of the pattern's source column (4-byte types), else a
-                    // synchronous copy; Constant: the constant
-#pragma unroll
-                    for (int c = 0; c < NIN; ++c) {
-                        T *dst = rb + (size_t)c * SW;
-                        if (MODE == CONSTANT && !rowok) {
-                            for (int x = lane; x < SW; x += 32) dst[x] = p.cval;
-                            continue;
-                        }
-                        const T *src = p.in[c] + (ptrdiff_t)yy * g.in_pitch;
-                        auto fix = [&](int x) {
-                            if constexpr (MODE == CONSTANT) {
-                                dst[x - XS] = (x >= 0 && x < g.w) ? __ldg(src + x) : p.cval;
-                            } else {
-                                const int xs = fixup_source<Op, MODE, CK>(x, g);
-                                if (xs < 0) return;
-                                if constexpr (ASYNC_FIX) cp_async4(dst + (x - XS), src + xs);
-                                else dst[x - XS] = __ldg(src + xs);
-                            }
-                        };
-                        if constexpr ((CK & CK_L) != 0)
-                            for (int x = XS + lane; x < cs; x += 32) fix(x);
-                        if constexpr ((CK & CK_R) != 0)
-                            for (int x = ce + lane; x < X0 + TW + HXA; x += 32) fix(x);
-                    }
-                }
-            }
-            if constexpr (ASYNC_FIX) cp_async_mbar_arrive_noinc(&full[s]);
-            if constexpr (MODE == CONSTANT && (CK & (CK_T | CK_B)) != 0)
-                fence_proxy_async();  // generic row fills before later bulk (async-proxy) writes
-            __syncwarp();
-            if (lane == 0) mbar_arrive(&full[s]);
-            if (++s == S) { s = 0; ph ^= 1; }
+        switch (g.mode) {  // the border pattern is a runtime parameter of the staged kernel
+        case CLAMP: staged_producer<Op, CLAMP, CK>(p, full, empty, buf, y0, nr, X0); break;
+        case MIRROR: staged_producer<Op, MIRROR, CK>(p, full, empty, buf, y0, nr, X0); break;
+        case REPEAT: staged_producer<Op, REPEAT, CK>(p, full, empty, buf, y0, nr, X0); break;
+        default: staged_producer<Op, CONSTANT, CK>(p, full, empty, buf, y0, nr, X0); break;
         }
         return;
     }
@@ -299,21 +321,21 @@ __device__ __forceinline__ void staged_body(const typename Op::Params &p, unsign
 
 // The TMA-staged fat kernel: Listing 3 on (blockIdx.x, blockIdx.y) with the staging
 // bounds of Geom (BH_L/BH_R from the aligned halo HXA, reading A21).
-template <class Op, int MODE>
+template <class Op>
 __global__ void __launch_bounds__(kStagedThreads) k_staged(const __grid_constant__ typename Op::Params p)
 {
     extern __shared__ __align__(128) unsigned char smem[];
     const int rg = region_of(p.g, blockIdx.x, blockIdx.y, 0, false);
     switch (rg) {
-    case RG_TL: staged_body<Op, MODE, region_checks(RG_TL)>(p, smem); break;
-    case RG_TR: staged_body<Op, MODE, region_checks(RG_TR)>(p, smem); break;
-    case RG_T: staged_body<Op, MODE, region_checks(RG_T)>(p, smem); break;
-    case RG_BL: staged_body<Op, MODE, region_checks(RG_BL)>(p, smem); break;
-    case RG_BR: staged_body<Op, MODE, region_checks(RG_BR)>(p, smem); break;
-    case RG_B: staged_body<Op, MODE, region_checks(RG_B)>(p, smem); break;
-    case RG_R: staged_body<Op, MODE, region_checks(RG_R)>(p, smem); break;
-    case RG_L: staged_body<Op, MODE, region_checks(RG_L)>(p, smem); break;
-    default: staged_body<Op, MODE, 0>(p, smem); break;
+    case RG_TL: staged_body<Op, region_checks(RG_TL)>(p, smem); break;
+    case RG_TR: staged_body<Op, region_checks(RG_TR)>(p, smem); break;
+    case RG_T: staged_body<Op, region_checks(RG_T)>(p, smem); break;
+    case RG_BL: staged_body<Op, region_checks(RG_BL)>(p, smem); break;
+    case RG_BR: staged_body<Op, region_checks(RG_BR)>(p, smem); break;
+    case RG_B: staged_body<Op, region_checks(RG_B)>(p, smem); break;
+    case RG_R: staged_body<Op, region_checks(RG_R)>(p, smem); break;
+    case RG_L: staged_body<Op, region_checks(RG_L)>(p, smem); break;
+    default: staged_body<Op, 0>(p, smem); break;
     }
 }
 

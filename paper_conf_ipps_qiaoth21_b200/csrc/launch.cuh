@@ -25,7 +25,7 @@ const void *kernel_for_disp(int disp)
     } else {
         switch (disp) {
         case DISP_TMA:
-            if constexpr (!Op::ROW_DIRECT) return (const void *)k_staged<Op, MODE>;
+            if constexpr (!Op::ROW_DIRECT) return (const void *)k_staged<Op>;  // one kernel, all modes
             else return nullptr;
         case DISP_BLOCK: return (const void *)k_stencil<Op, MODE, DISP_BLOCK>;
         case DISP_WARP: return (const void *)k_stencil<Op, MODE, DISP_BLOCK>;

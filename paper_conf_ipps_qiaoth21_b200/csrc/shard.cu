@@ -38,14 +38,18 @@ template <class T> ncclDataType_t nccl_type();
 template <> ncclDataType_t nccl_type<float>() { return ncclFloat32; }
 template <> ncclDataType_t nccl_type<uint8_t>() { return ncclUint8; }
 
+// ctx == nullptr: local mode (no exchange; the caller filled the halo rows).
 template <class T, class F>
-isp_status_t shard_run(isp_shard_ctx *ctx, T *strip, int w, int H, int pitch, int halo, int hy, int mode,
-                       T *out, int out_pitch, cudaStream_t stream, cudaStream_t comm, F &&filter_rows)
+isp_status_t shard_run(isp_shard_ctx *ctx, int rank, int nranks, T *strip, int w, int H, int pitch, int halo,
+                       int hy, int mode, T *out, int out_pitch, cudaStream_t stream, cudaStream_t comm,
+                       F &&filter_rows)
 {
+    (void)w;
     isp_shard_sched sc;
-    isp_status_t s = isp_shard_schedule(H, ctx->rank, ctx->nranks, halo, hy, mode, &sc);
+    isp_status_t s = isp_shard_schedule(H, rank, nranks, halo, hy, mode, &sc);
     if (s != ISP_OK) return s;
-    if (cudaSetDevice(ctx->device) != cudaSuccess) return ispi_fail(ISP_ECUDA, "cudaSetDevice");
+    if (!ctx) sc.n_ops = 0;
+    if (ctx && cudaSetDevice(ctx->device) != cudaSuccess) return ispi_fail(ISP_ECUDA, "cudaSetDevice");
     const size_t row_elems = (size_t)pitch;
     if (sc.n_ops > 0) {
         if (cudaEventRecord(ctx->ev_ready, stream) != cudaSuccess ||
@@ -180,6 +184,19 @@ isp_status_t isp_shard_init(isp_shard_ctx **ctx, const unsigned char id[128], in
     return ISP_OK;
 }
 
+isp_status_t isp_shard_filter_local_f32(float *strip, int w, int H, int pitch, int halo, int rank, int nranks,
+                                        const float *mask, int mw, int mh, int border_mode, float const_val,
+                                        float *out, int out_pitch, isp_variant_t variant, isp_stream_t stream)
+{
+    if (!strip || !out || !mask) return ispi_fail(ISP_EINVAL, "null pointer");
+    auto f = [&](const float *in_base, float *o, const RowRange &rr) {
+        return ispi_filter_f32(in_base, w, H, pitch, mask, mw, mh, border_mode, const_val, o, out_pitch, variant,
+                               stream, &rr);
+    };
+    return shard_run<float>(nullptr, rank, nranks, strip, w, H, pitch, halo, mh / 2, border_mode, out, out_pitch,
+                            (cudaStream_t)stream, (cudaStream_t)stream, f);
+}
+
 isp_status_t isp_shard_destroy(isp_shard_ctx *ctx)
 {
     if (!ctx) return ISP_OK;
@@ -199,8 +216,8 @@ isp_status_t isp_shard_filter_f32(isp_shard_ctx *ctx, float *strip, int w, int H
         return ispi_filter_f32(in_base, w, H, pitch, mask, mw, mh, border_mode, const_val, o, out_pitch, variant,
                                stream, &rr);
     };
-    return shard_run<float>(ctx, strip, w, H, pitch, halo, mh / 2, border_mode, out, out_pitch, (cudaStream_t)stream,
-                            (cudaStream_t)comm_stream, f);
+    return shard_run<float>(ctx, ctx->rank, ctx->nranks, strip, w, H, pitch, halo, mh / 2, border_mode, out, out_pitch,
+                            (cudaStream_t)stream, (cudaStream_t)comm_stream, f);
 }
 
 isp_status_t isp_shard_filter_u8(isp_shard_ctx *ctx, uint8_t *strip, int w, int H, int pitch, int halo,
@@ -213,8 +230,8 @@ isp_status_t isp_shard_filter_u8(isp_shard_ctx *ctx, uint8_t *strip, int w, int 
         return ispi_filter_u8(in_base, w, H, pitch, mask, mw, mh, divisor, border_mode, const_val, o, out_pitch,
                               variant, stream, &rr);
     };
-    return shard_run<uint8_t>(ctx, strip, w, H, pitch, halo, mh / 2, border_mode, out, out_pitch,
-                              (cudaStream_t)stream, (cudaStream_t)comm_stream, f);
+    return shard_run<uint8_t>(ctx, ctx->rank, ctx->nranks, strip, w, H, pitch, halo, mh / 2, border_mode, out,
+                              out_pitch, (cudaStream_t)stream, (cudaStream_t)comm_stream, f);
 }
 
 }  // extern "C"

@@ -29,6 +29,7 @@ def main():
     ap.add_argument("--window", type=int, default=5)
     ap.add_argument("--env", action="append", default=[""])
     ap.add_argument("--override", action="append", default=[], help="WX,TY launch override settings")
+    ap.add_argument("--cycle", action="store_true", help="cycle the four border modes inside the graph")
     a = ap.parse_args()
     n = a.size
     b = synth.binomial_row(a.window).astype(np.float64)
@@ -48,9 +49,12 @@ def main():
             isp.isp_set_launch_override(wx, ty)
         R, reps = 12, 40
 
+        modes = ["clamp", "mirror", "repeat", "constant"]
+
         def launch(i):
             inp, out = pairs[i % 6]
-            isp.isp_filter_ex(inp, mask, a.mode, 0.5, out=out, variant=a.variant, stream=stream)
+            m = modes[i % 4] if a.cycle else a.mode
+            isp.isp_filter_ex(inp, mask, m, 0.5, out=out, variant=a.variant, stream=stream)
 
         with torch.cuda.stream(stream):
             for i in range(3):
@@ -70,7 +74,8 @@ def main():
             e1.record(stream)
         torch.cuda.synchronize()
         us = 1e3 * e0.elapsed_time(e1) / (R * reps)
-        print(json.dumps({"env": env, "override": ov, "variant": a.variant, "mode": a.mode, "us": round(us, 3),
+        print(json.dumps({"env": env, "override": ov, "variant": a.variant, "mode": "cycle" if a.cycle else a.mode,
+                          "us": round(us, 3),
                           "gbs": round(8 * n * n / (us * 1e-6) / 1e9, 1),
                           "plan": {k: plan[k] for k in ("tile_w", "tile_h", "nx", "ny", "choice")}}), flush=True)
         for k in keys:

@@ -33,7 +33,7 @@ METRICS = [
 ]
 
 UNIT_SCALE = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "nsecond": 1e-3, "usecond": 1.0,
-              "msecond": 1e3}
+              "msecond": 1e3, "ns": 1e-3, "us": 1.0, "ms": 1e3}
 
 
 def raw_rows(rep):
@@ -54,7 +54,7 @@ def raw_rows(rep):
                 if u in ("byte", "Kbyte", "Mbyte", "Gbyte"):
                     v *= UNIT_SCALE[u]
                     m = m + " [bytes]"
-                elif u in ("nsecond", "usecond", "msecond"):
+                elif u in ("nsecond", "usecond", "msecond", "ns", "us", "ms"):
                     v *= UNIT_SCALE[u]
                     m = m + " [us]"
                 d[m] = v
