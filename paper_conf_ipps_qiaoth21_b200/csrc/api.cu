@@ -335,7 +335,10 @@ isp_status_t resolve_and_launch(Desc &d, int fam, int w, int h, int mw, int mh, 
 
     isp_variant_t chosen = v;
     if (chosen == ISP_TMA && !tma_ok) chosen = ISP_BLOCK;      // misaligned / not built: streaming
-    if (v == ISP_AUTO) chosen = tma_ok ? ISP_TMA : (p0.wx > 1 ? ISP_WARP : ISP_BLOCK);
+    // AUTO's ISP kernel: TMA-staged for 4-byte pixels; for sub-word pixels (u8, i16) the
+    // staged L/R CTAs fix up their halo synchronously, so the streaming Listing-5 kernel
+    // is faster there (measured, profiles/r01_suite.json cfg3)
+    if (v == ISP_AUTO) chosen = (tma_ok && esz == 4) ? ISP_TMA : (p0.wx > 1 ? ISP_WARP : ISP_BLOCK);
     auto plan_for = [&](isp_variant_t c) {
         if (c == ISP_TMA) {
             Plan q = make_plan(w, h, hx, hy, px, STAGED_WARPS * 32 * px, 0, 0, rr, nb_tma);
@@ -344,7 +347,11 @@ isp_status_t resolve_and_launch(Desc &d, int fam, int w, int h, int mw, int mh, 
         }
         // streaming / naive kernels: uniform tiles of kStreamTileRows rows (Eq. 2 verbatim);
         // several waves of small blocks hide their load latency best (measured)
-        return make_plan(w, h, hx, hy, px, 0, g_override_ty > 0 ? 0 : kStreamTileRows, 0, rr,
+        // small images: shorter tiles so the grid still covers the SMs (latency-bound)
+        int ty = kStreamTileRows;
+        const int nrw = rr ? rr->nrows : h;
+        while (ty > 1 && (long long)p0.nx * ceil_div(nrw, ty) < num_sms()) ty /= 2;
+        return make_plan(w, h, hx, hy, px, 0, g_override_ty > 0 ? 0 : ty, 0, rr,
                          c == ISP_NAIVE ? nb_naive : nb_stream);
     };
     Plan p = plan_for(chosen);

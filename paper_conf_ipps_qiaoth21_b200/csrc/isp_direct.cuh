@@ -58,6 +58,8 @@ __device__ __forceinline__ void direct_body(const typename Op::Params &p, int x0
 template <class Op, int MODE, int DISP>
 __global__ void __launch_bounds__(256) k_direct(const __grid_constant__ typename Op::Params p)
 {
+    pdl_launch_dependents();
+    pdl_wait();
     const int lane = threadIdx.x & 31;
     const int warp = threadIdx.x >> 5;
     const int nwarp = blockDim.x >> 5;

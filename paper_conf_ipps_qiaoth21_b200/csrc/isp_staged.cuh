@@ -259,6 +259,7 @@ __device__ __forceinline__ void staged_body(const typename Op::Params &p, unsign
         fence_mbar_init();
     }
     __syncthreads();
+    pdl_wait();  // the prologue above overlaps the previous kernel's tail (PDL)
 
     if (warp == NWC) {
         switch (g.mode) {  // the border pattern is a runtime parameter of the staged kernel
@@ -325,6 +326,7 @@ template <class Op>
 __global__ void __launch_bounds__(kStagedThreads) k_staged(const __grid_constant__ typename Op::Params p)
 {
     extern __shared__ __align__(128) unsigned char smem[];
+    pdl_launch_dependents();
     const int rg = region_of(p.g, blockIdx.x, blockIdx.y, 0, false);
     switch (rg) {
     case RG_TL: staged_body<Op, region_checks(RG_TL)>(p, smem); break;

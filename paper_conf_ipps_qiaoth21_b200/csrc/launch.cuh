@@ -1,5 +1,6 @@
 // launch.cuh -- template glue: pick the (op, mode, dispatch) kernel instance and launch it.
 #pragma once
+#include <cstdlib>
 #include <mutex>
 #include <unordered_map>
 
@@ -49,6 +50,15 @@ const void *kernel_for(int mode, int disp)
     return nullptr;
 }
 
+inline bool pdl_enabled()
+{
+    static const bool on = [] {
+        const char *e = getenv("ISP_PDL");
+        return !(e && e[0] == '0');
+    }();
+    return on;
+}
+
 template <class P>
 cudaError_t launch_params(const void *fn, const Desc &d, const P &p)
 {
@@ -65,7 +75,19 @@ cudaError_t launch_params(const void *fn, const Desc &d, const P &p)
         }
     }
     void *args[] = {const_cast<P *>(&p)};
-    return cudaLaunchKernel(fn, d.grid, d.block, args, d.smem, d.stream);
+    // programmatic dependent launch: the kernels call griddepcontrol.wait before touching
+    // global memory, so their launch/prologue may overlap the previous kernel's tail
+    cudaLaunchConfig_t cfg{};
+    cfg.gridDim = d.grid;
+    cfg.blockDim = d.block;
+    cfg.dynamicSmemBytes = d.smem;
+    cfg.stream = d.stream;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = pdl_enabled() ? 1 : 0;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    return cudaLaunchKernelExC(&cfg, fn, args);
 }
 
 }  // namespace ispk
