@@ -119,10 +119,11 @@ def lib():
     """Load libisp.so (the CUDA path).  Raises ImportError if it is not built."""
     global _lib
     if _lib is None:
-        if not os.path.exists(LIB_PATH):
-            raise ImportError(f"{LIB_PATH} missing: run `python -m paper_conf_ipps_qiaoth21_b200.build` "
+        path = os.environ.get("ISP_LIB_PATH") or LIB_PATH  # experiment builds (tools/exp_lib.py)
+        if not os.path.exists(path):
+            raise ImportError(f"{path} missing: run `python -m paper_conf_ipps_qiaoth21_b200.build` "
                               "(there is no CPU fallback)")
-        L = ctypes.CDLL(LIB_PATH)
+        L = ctypes.CDLL(path)
         for name, args in _SIGS.items():
             f = getattr(L, name)
             f.argtypes = args

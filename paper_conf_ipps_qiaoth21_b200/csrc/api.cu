@@ -24,6 +24,15 @@ thread_local char g_err[512] = "";
 thread_local isp_plan_info g_last_plan{};
 int g_override_wx = 0, g_override_ty = 0;
 
+// Rows of the strips holding the image's top / bottom border in a balanced split, in
+// 1/256 of an interior strip (0 = uniform); ISP_EDGE_W overrides.
+constexpr int kEdgeW = 64;
+int edge_w_setting()
+{
+    const char *e = getenv("ISP_EDGE_W");
+    return e ? std::max(0, atoi(e)) : kEdgeW;
+}
+
 }  // namespace
 
 isp_status_t ispi_fail(isp_status_t s, const char *fmt, ...)
@@ -73,6 +82,7 @@ struct Plan {
     int px, wx, ty, tile_w, warp_w;
     int nx, ny;
     int bh_l, bh_r, bh_t, bh_b, w_l, w_r;
+    int edge_w;  // balanced split: weight of the image's first / last strip (x 1/256)
     bool degenerate;
 };
 
@@ -144,7 +154,15 @@ Plan make_plan(int w, int h, int hx, int hy, int px, int tile_w_req, int tile_h_
     } else {
         // same definition on the balanced split: first block row whose reads stay >= 0,
         // first block row whose reads reach past the image bottom
-        auto y0_of = [&](long long by) { return rr->oy0 + (by * nr) / p.ny; };
+        // (block_rows in isp_core.cuh: border strips weighted by edge_w / 256)
+        p.edge_w = p.ny > 2 ? edge_w_setting() : 0;
+        const long long ft = rr->t_real ? p.edge_w : 256, fb = rr->b_real ? p.edge_w : 256;
+        const long long W = ft + fb + 256ll * (p.ny - 2);
+        auto y0_of = [&](long long by) {
+            if (p.edge_w <= 0) return rr->oy0 + (by * nr) / p.ny;
+            const long long c = by == 0 ? 0 : by == p.ny ? W : ft + 256ll * (by - 1);
+            return rr->oy0 + (c * nr) / W;
+        };
         int bt = 0;
         if (rr->t_real)
             while (bt < p.ny && y0_of(bt) - hy < 0) ++bt;
@@ -302,6 +320,16 @@ void apply_staged_bounds(Plan &p, int w, int px, const StagedGeom &sg)
     p.degenerate = p.bh_l > p.bh_r || p.bh_t > p.bh_b;
 }
 
+// Diagnostics: per-CTA timestamps of TMA-staged launches (env ISP_CTA_TRACE), 4 words
+// per CTA, read back with isp_debug_cta_trace.
+constexpr int kTraceCtas = 1 << 16;
+unsigned long long *cta_trace_buffer()
+{
+    static unsigned long long *buf = nullptr;
+    if (!buf && cudaMalloc(&buf, sizeof(unsigned long long) * 4 * kTraceCtas) != cudaSuccess) buf = nullptr;
+    return buf;
+}
+
 // Resolve the variant (AUTO = "isp+m") and launch.  tma_ok: the op has a staged
 // kernel and the input rows are 16-B aligned; esz / nin: input element size / count.
 isp_status_t resolve_and_launch(Desc &d, int fam, int w, int h, int mw, int mh, int hx, int hy, bool direct,
@@ -395,6 +423,8 @@ isp_status_t resolve_and_launch(Desc &d, int fam, int w, int h, int mw, int mh, 
     d.g.warp_level = chosen == ISP_WARP;
     d.g.mode = d.mode;
     if (const char *e = getenv("ISP_DEBUG_STAGED")) d.g.dbg = atoi(e);
+    if (getenv("ISP_CTA_TRACE")) d.g.trace = cta_trace_buffer();
+    d.g.edge_w = p.edge_w;
     g_last_plan = info;
     cudaError_t e = run(d);
     if (e == cudaSuccess) e = cudaGetLastError();
@@ -506,6 +536,16 @@ const char *isp_status_string(isp_status_t s)
 
 const char *isp_last_error(void) { return g_err; }
 int isp_version(void) { return 1; }
+
+/* Diagnostics (not part of the contract): copy the per-CTA trace of the last TMA-staged
+ * launches made with ISP_CTA_TRACE set (n CTAs x {smid|region<<16|by<<32|bx<<48, t0, t1, 0}). */
+int isp_debug_cta_trace(unsigned long long *host, int n)
+{
+    unsigned long long *b = cta_trace_buffer();
+    if (!b || n < 0 || n > kTraceCtas) return ISP_EINVAL;
+    return cudaMemcpy(host, b, sizeof(unsigned long long) * 4 * (size_t)n, cudaMemcpyDeviceToHost) == cudaSuccess
+               ? ISP_OK : ISP_ECUDA;
+}
 
 isp_status_t isp_last_plan(isp_plan_info *out)
 {

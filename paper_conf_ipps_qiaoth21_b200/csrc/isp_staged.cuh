@@ -260,6 +260,7 @@ __device__ __forceinline__ void staged_body(const typename Op::Params &p, unsign
     }
     __syncthreads();
     pdl_wait();  // the prologue above overlaps the previous kernel's tail (PDL)
+    if (g.trace && threadIdx.x == 0) g.trace[4ull * (blockIdx.y * gridDim.x + blockIdx.x) + 3] = gtimer();
 
     if (warp == NWC) {
         switch (g.mode) {  // the border pattern is a runtime parameter of the staged kernel
@@ -328,6 +329,7 @@ __global__ void __launch_bounds__(kStagedThreads) k_staged(const __grid_constant
     extern __shared__ __align__(128) unsigned char smem[];
     pdl_launch_dependents();
     const int rg = region_of(p.g, blockIdx.x, blockIdx.y, 0, false);
+    const unsigned long long t0 = p.g.trace ? gtimer() : 0;
     switch (rg) {
     case RG_TL: staged_body<Op, region_checks(RG_TL)>(p, smem); break;
     case RG_TR: staged_body<Op, region_checks(RG_TR)>(p, smem); break;
@@ -338,6 +340,13 @@ __global__ void __launch_bounds__(kStagedThreads) k_staged(const __grid_constant
     case RG_R: staged_body<Op, region_checks(RG_R)>(p, smem); break;
     case RG_L: staged_body<Op, region_checks(RG_L)>(p, smem); break;
     default: staged_body<Op, 0>(p, smem); break;
+    }
+    if (p.g.trace && threadIdx.x == 0) {  // compute warp 0 finished its rows
+        unsigned long long *t = p.g.trace + 4ull * (blockIdx.y * gridDim.x + blockIdx.x);
+        t[0] = (unsigned long long)smid() | ((unsigned long long)rg << 16) | ((unsigned long long)blockIdx.y << 32) |
+               ((unsigned long long)blockIdx.x << 48);
+        t[1] = t0;
+        t[2] = gtimer();
     }
 }
 

@@ -1,0 +1,38 @@
+#!/usr/bin/env python
+"""A few plain launches of one filter call, for ncu captures (no graphs, no timing).
+
+    ncu --set full -k regex:k_staged -s 2 -c 1 python tools/prof_one.py --variant tma --mode clamp
+"""
+import argparse
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+
+import numpy as np  # noqa: E402
+import torch  # noqa: E402
+
+import paper_conf_ipps_qiaoth21_b200 as isp  # noqa: E402
+import synth  # noqa: E402
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--variant", default="tma")
+    ap.add_argument("--mode", default="clamp")
+    ap.add_argument("--size", type=int, default=4096)
+    ap.add_argument("--window", type=int, default=5)
+    ap.add_argument("--launches", type=int, default=4)
+    a = ap.parse_args()
+    n = a.size
+    b = synth.binomial_row(a.window).astype(np.float64)
+    mask = (np.outer(b, b) / b.sum() ** 2).astype(np.float32)
+    inp = torch.from_numpy(synth.uniform_f32(n, n, 2)).cuda()
+    out = torch.empty_like(inp)
+    for _ in range(a.launches):
+        isp.isp_filter_ex(inp, mask, a.mode, 0.5, out=out, variant=a.variant)
+    torch.cuda.synchronize()
+
+
+if __name__ == "__main__":
+    main()
