@@ -43,6 +43,7 @@ struct OpConvF32 {
     static constexpr int NIN = 1, PX = 4, HX = MW_ / 2, HY = MH_ / 2, MH = MH_, SEGW = PX + 2 * HX;
     static constexpr int PFMAX = 0;
     static constexpr bool ROW_DIRECT = false;
+    static constexpr bool SHFL_HALO = false;  // shuffle halo measured slower
     struct Params {
         Geom g;
         const float *in[1];
@@ -92,6 +93,7 @@ struct OpSepF32 {
     static constexpr int NIN = 1, PX = 4, HX = MW_ / 2, HY = MH_ / 2, MH = MH_, SEGW = PX + 2 * HX;
     static constexpr int PFMAX = 0;
     static constexpr bool ROW_DIRECT = false;
+    static constexpr bool SHFL_HALO = false;  // shuffle halo measured slower
     struct Params {
         Geom g;
         const float *in[1];
@@ -158,9 +160,10 @@ __device__ __forceinline__ uint8_t sat_u8(int v) { return (uint8_t)min(255, max(
 template <int MW_, int MH_>
 struct OpConvU8 {
     using Tin = uint8_t;
-    static constexpr int NIN = 1, PX = 8, HX = MW_ / 2, HY = MH_ / 2, MH = MH_, SEGW = PX + 2 * HX;
+    static constexpr int NIN = 1, PX = kPxU8, HX = MW_ / 2, HY = MH_ / 2, MH = MH_, SEGW = PX + 2 * HX;
     static constexpr int PFMAX = 0;
     static constexpr bool ROW_DIRECT = false;
+    static constexpr bool SHFL_HALO = false;  // shuffle halo measured slower
     struct Params {
         Geom g;
         const uint8_t *in[1];
@@ -206,9 +209,10 @@ struct OpConvU8 {
 template <int MW_, int MH_>
 struct OpSepU8 {
     using Tin = uint8_t;
-    static constexpr int NIN = 1, PX = 8, HX = MW_ / 2, HY = MH_ / 2, MH = MH_, SEGW = PX + 2 * HX;
+    static constexpr int NIN = 1, PX = kPxU8, HX = MW_ / 2, HY = MH_ / 2, MH = MH_, SEGW = PX + 2 * HX;
     static constexpr int PFMAX = 0;
     static constexpr bool ROW_DIRECT = false;
+    static constexpr bool SHFL_HALO = false;  // shuffle halo measured slower
     struct Params {
         Geom g;
         const uint8_t *in[1];
@@ -253,15 +257,17 @@ struct OpSepU8 {
     }
 };
 
-// Exact round-half-up integer square root for n < 2^24 (Sobel magnitude, a9):
-// floor via correctly-rounded sqrtf (n exact in f32) + correction, then +1 iff n - r^2 > r.
-__device__ __forceinline__ int isqrt_round(int n)
+// Sobel magnitude min(255, round_half_up(sqrt(n))) for integer n >= 0 (a9), exact:
+// for n <= 65280 (= 255.5^2 - 0.25, beyond which the result saturates to 255) sqrt(n)
+// stays >= 1.5e-3 from every integer - 1/2 (n and k^2 +- k are integers), while
+// sqrt.approx.f32 errs by a few ulp (< 1e-4 at 255.5), so floor(sqrt(n) + 1/2) taken in
+// f32 is the exact rounding.
+__device__ __forceinline__ int sobel_mag(int n)
 {
-    int r = (int)sqrtf((float)n);
-    if (r * r > n) --r;
-    if ((r + 1) * (r + 1) <= n) ++r;
-    if (n - r * r > r) ++r;
-    return r;
+    const float f = (float)min(n, 65280);
+    float r;
+    asm("sqrt.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(f));
+    return (int)(r + 0.5f);
 }
 
 // ---------------------------------------------------------------------------------
@@ -270,9 +276,10 @@ __device__ __forceinline__ int isqrt_round(int n)
 // ---------------------------------------------------------------------------------
 struct OpSobel {
     using Tin = uint8_t;
-    static constexpr int NIN = 1, PX = 8, HX = 1, HY = 1, MH = 3, SEGW = PX + 2;
+    static constexpr int NIN = 1, PX = kPxU8, HX = 1, HY = 1, MH = 3, SEGW = PX + 2;
     static constexpr int PFMAX = 0;
     static constexpr bool ROW_DIRECT = false;
+    static constexpr bool SHFL_HALO = false;  // shuffle halo measured slower
     struct Params {
         Geom g;
         const uint8_t *in[1];
@@ -328,7 +335,7 @@ struct OpSobel {
             uint8_t o[PX];
 #pragma unroll
             for (int e = 0; e < PX; ++e)
-                o[e] = (uint8_t)min(255, isqrt_round(a.v[0][e] * a.v[0][e] + a.v[1][e] * a.v[1][e]));
+                o[e] = (uint8_t)sobel_mag(a.v[0][e] * a.v[0][e] + a.v[1][e] * a.v[1][e]);
             store_px<CK, uint8_t, PX>(p.mag + off, x0, p.g.w, p.g.vec_out, o);
         }
     }
@@ -337,9 +344,10 @@ struct OpSobel {
 // Laplace 5x5 (a8): box sum minus 25 x centre (== ones mask with centre -24).
 struct OpLaplace5 {
     using Tin = uint8_t;
-    static constexpr int NIN = 1, PX = 8, HX = 2, HY = 2, MH = 5, SEGW = PX + 4;
+    static constexpr int NIN = 1, PX = kPxU8, HX = 2, HY = 2, MH = 5, SEGW = PX + 4;
     static constexpr int PFMAX = 0;
     static constexpr bool ROW_DIRECT = false;
+    static constexpr bool SHFL_HALO = false;  // shuffle halo measured slower
     struct Params {
         Geom g;
         const uint8_t *in[1];
@@ -392,6 +400,7 @@ struct OpHarris {
     static constexpr int NIN = 2, PX = 4, HX = 1, HY = 1, MH = 3, SEGW = PX + 2;
     static constexpr int PFMAX = 0;
     static constexpr bool ROW_DIRECT = false;
+    static constexpr bool SHFL_HALO = false;  // shuffle halo measured slower
     struct Params {
         Geom g;
         const int16_t *in[2];
@@ -460,6 +469,7 @@ struct OpAtrous {
     static constexpr int NIN = 1, PX = 4, HX = D, HY = D, MH = 2 * D + 1, SEGW = PX + 2 * D;
     static constexpr int PFMAX = 0;
     static constexpr bool ROW_DIRECT = true;
+    static constexpr bool SHFL_HALO = false;
     static constexpr int NTAPS_Y = 3;
     __host__ __device__ static constexpr int vtap(int t) { return (t - 1) * D; }
     struct Params {

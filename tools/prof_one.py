@@ -23,8 +23,28 @@ def main():
     ap.add_argument("--size", type=int, default=4096)
     ap.add_argument("--window", type=int, default=5)
     ap.add_argument("--launches", type=int, default=4)
+    ap.add_argument("--op", default="gauss", choices=["gauss", "sobel", "laplace", "harris", "bilateral"])
     a = ap.parse_args()
     n = a.size
+    if a.op != "gauss":
+        u8 = torch.from_numpy(synth.uniform_u8(n, n, 3)).cuda()
+        dx = torch.empty((n, n), dtype=torch.int16, device="cuda")
+        dy = torch.empty_like(dx)
+        o8 = torch.empty_like(u8)
+        f = torch.from_numpy(synth.uniform_f32(n, n, 4)).cuda()
+        fo = torch.empty_like(f)
+        isp.isp_sobel_u8(u8, a.mode, dx=dx, dy=dy, mag=o8)
+        for _ in range(a.launches):
+            if a.op == "sobel":
+                isp.isp_sobel_u8(u8, a.mode, dx=dx, dy=dy, mag=o8, variant=a.variant)
+            elif a.op == "laplace":
+                isp.isp_laplace5_u8(u8, a.mode, out=o8, variant=a.variant)
+            elif a.op == "harris":
+                isp.isp_harris_u8(dx, dy, a.mode, out=o8, variant=a.variant)
+            else:
+                isp.isp_bilateral_f32(f, a.window, (a.window - 1) / 4.0, 0.1, a.mode, 0.5, out=fo, variant=a.variant)
+        torch.cuda.synchronize()
+        return
     b = synth.binomial_row(a.window).astype(np.float64)
     mask = (np.outer(b, b) / b.sum() ** 2).astype(np.float32)
     inp = torch.from_numpy(synth.uniform_f32(n, n, 2)).cuda()
