@@ -354,10 +354,15 @@ isp_status_t resolve_and_launch(Desc &d, int fam, int w, int h, int mw, int mh, 
         return kfn(q);
     };
     const StagedGeom sg = staged_geom(w, hx, hy, px, esz, nin);
-    tma_ok = tma_ok && !direct && fn_of(DISP_TMA) != nullptr && g_override_wx == 0;
+    // runtime-window (direct) ops: the staged variant is the shared-memory tiled kernel
+    // (isp_direct.cuh k_tile), which needs no alignment
+    if (direct) tma_ok = true;
+    tma_ok = tma_ok && fn_of(DISP_TMA) != nullptr && g_override_wx == 0;
+    const int tma_threads = direct ? TILE_THREADS : STAGED_THREADS;
+    const size_t tma_smem = direct ? (size_t)(TILE_PX * 32 + 2 * hx) * (TILE_H + 2 * hy) * esz : sg.smem;
     const int nb_naive = blocks_per_sm(fn_of(naive_disp), threads);
     const int nb_stream = blocks_per_sm(fn_of(p0.wx > 1 ? DISP_WARP : DISP_BLOCK), threads);
-    int nb_tma = tma_ok ? blocks_per_sm(fn_of(DISP_TMA), STAGED_THREADS, sg.smem) : 0;
+    int nb_tma = tma_ok ? blocks_per_sm(fn_of(DISP_TMA), tma_threads, tma_smem) : 0;
     if (const char *e = getenv("ISP_CTAS_PER_SM")) nb_tma = std::min(nb_tma, std::max(1, atoi(e)));
     if (tma_ok && nb_tma <= 0) tma_ok = false;
 
@@ -368,6 +373,8 @@ isp_status_t resolve_and_launch(Desc &d, int fam, int w, int h, int mw, int mh, 
     // is faster there (measured, profiles/r01_suite.json cfg3)
     if (v == ISP_AUTO) chosen = (tma_ok && esz == 4) ? ISP_TMA : (p0.wx > 1 ? ISP_WARP : ISP_BLOCK);
     auto plan_for = [&](isp_variant_t c) {
+        if (c == ISP_TMA && direct)  // tiles of TILE_PX*32 x TILE_H, Eq. (2) verbatim
+            return make_plan(w, h, hx, hy, px, TILE_PX * 32, TILE_H, TILE_PX * 32, rr, nb_tma);
         if (c == ISP_TMA) {
             Plan q = make_plan(w, h, hx, hy, px, STAGED_WARPS * 32 * px, 0, 0, rr, nb_tma);
             apply_staged_bounds(q, w, px, sg);
@@ -389,7 +396,7 @@ isp_status_t resolve_and_launch(Desc &d, int fam, int w, int h, int mw, int mh, 
         isp_model_params mp;
         defaults(fam, d.mode, mp);
         info.o_naive = nb_naive > 0 ? occupancy_of(nb_naive, threads) : 1.0;
-        info.o_isp = chosen == ISP_TMA ? occupancy_of(nb_tma, STAGED_THREADS)
+        info.o_isp = chosen == ISP_TMA ? occupancy_of(nb_tma, tma_threads)
                                        : (nb_stream > 0 ? occupancy_of(nb_stream, threads) : 1.0);
         n_block(p, info.n_block);
         model(p, w, h, mw, mh, mp, info);
@@ -409,8 +416,8 @@ isp_status_t resolve_and_launch(Desc &d, int fam, int w, int h, int mw, int mh, 
     d.g.stages = sg.stages;
     d.g.rs = sg.rs;
     d.grid = dim3(p.nx, p.ny, 1);
-    d.block = dim3(chosen == ISP_TMA ? STAGED_THREADS : threads, 1, 1);
-    d.smem = chosen == ISP_TMA ? sg.smem : 0;
+    d.block = dim3(chosen == ISP_TMA ? tma_threads : threads, 1, 1);
+    d.smem = chosen == ISP_TMA ? tma_smem : 0;
     info.bh_l = p.bh_l; info.bh_r = p.bh_r; info.bh_t = p.bh_t; info.bh_b = p.bh_b;
     info.nx = p.nx; info.ny = p.ny; info.w_l = p.w_l; info.w_r = p.w_r;
     info.degenerate = p.degenerate;

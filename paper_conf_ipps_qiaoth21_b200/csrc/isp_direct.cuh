@@ -9,6 +9,7 @@
 // window column, so one load serves PX taps.
 #pragma once
 #include "isp_ops.cuh"
+#include "kernels.h"
 
 namespace ispk {
 
@@ -88,11 +89,107 @@ __global__ void __launch_bounds__(256) k_direct(const __grid_constant__ typename
     }
 }
 
+// ---------------------------------------------------------------------------------
+// Shared-memory tiled form of the direct family (variant ISP_TMA for runtime-window ops:
+// the staged family of the expensive kernels).  CTA = kTileWarps warps over a tile of
+// kTileW x kTileH outputs; each thread owns PX outputs of one row at a stride of 32
+// columns, so a tap reads PX conflict-free words of one smem row and no value is moved
+// between taps.  ISP lives in the fill (reading A21): the CTA's region (Listing 3 on
+// the tile grid, Eq. 2 with this tile shape) decides which sides of the (tile + halo)
+// fill go through the border pattern; a Body CTA copies unchecked.  The compute loop
+// has no checks in any region and runs the same per-output operations in the same
+// order as direct_body, so all variants give identical bits.
+// ---------------------------------------------------------------------------------
+constexpr int kTileWarps = TILE_THREADS / 32, kTileThreads = TILE_THREADS, kTileH = TILE_H;
+
+template <class Op, int MODE, int CK>
+__device__ __forceinline__ void tile_fill(const typename Op::Params &p, typename Op::Tin *tile, int X0, int Y0,
+                                          int SW, int SH)
+{
+    using T = typename Op::Tin;
+    const Geom &g = p.g;
+    const int hx = p.mw / 2, hy = p.mh / 2;
+    for (int r = threadIdx.x / 32; r < SH; r += kTileWarps) {
+        bool rowok;
+        const int yy = map_row<MODE, CK>(Y0 - hy + r, g, rowok);
+        const T *__restrict__ row = p.in + (ptrdiff_t)yy * g.in_pitch;
+        T *dst = tile + r * SW;
+        for (int c = threadIdx.x & 31; c < SW; c += 32) {
+            const int x = X0 - hx + c;
+            if constexpr ((CK & (CK_L | CK_R | CK_T | CK_B)) == 0) {
+                dst[c] = __ldg(row + x);                       // Body: no checks
+            } else {
+                dst[c] = load_x<T, MODE, CK>(row, rowok, x, g, p.cval);
+            }
+        }
+    }
+}
+
+template <class Op, int MODE, int CK>
+__device__ __forceinline__ void tile_body(const typename Op::Params &p, typename Op::Tin *tile)
+{
+    using T = typename Op::Tin;
+    constexpr int PX = Op::PX, TW = 32 * PX;
+    static_assert(PX == TILE_PX, "the planner sizes tiles with TILE_PX");
+    const int X0 = blockIdx.x * TW, Y0 = p.g.oy0 + blockIdx.y * kTileH;
+    const int SW = TW + 2 * (p.mw / 2), SH = kTileH + 2 * (p.mh / 2);
+    tile_fill<Op, MODE, CK>(p, tile, X0, Y0, SW, SH);
+    __syncthreads();
+    const int lane = threadIdx.x & 31;
+    for (int o = threadIdx.x / 32; o < kTileH; o += kTileWarps) {
+        const int y = Y0 + o;
+        if ((CK & CK_B) && y >= p.g.y_end) break;
+        typename Op::A acc;
+        Op::init_tile(p, acc, tile + (o + p.mh / 2) * SW + p.mw / 2 + lane);
+        for (int j = 0; j < p.mh; ++j) {
+            const T *srow = tile + (o + j) * SW + lane;
+#pragma unroll 2
+            for (int i = 0; i < p.mw; ++i) {
+                T win[PX];
+#pragma unroll
+                for (int e = 0; e < PX; ++e) win[e] = srow[i + 32 * e];
+                Op::tap(p, j, i, win, acc);
+            }
+        }
+        Op::template store_strided<CK>(p, acc, X0 + lane, y);
+    }
+}
+
+template <class Op, int MODE>
+__global__ void __launch_bounds__(kTileThreads) k_tile(const __grid_constant__ typename Op::Params p)
+{
+    extern __shared__ __align__(16) unsigned char tile_smem[];
+    auto *tile = reinterpret_cast<typename Op::Tin *>(tile_smem);
+    pdl_launch_dependents();
+    pdl_wait();
+    switch (region_of(p.g, blockIdx.x, blockIdx.y, 0, false)) {
+    case RG_TL: tile_body<Op, MODE, region_checks(RG_TL)>(p, tile); break;
+    case RG_TR: tile_body<Op, MODE, region_checks(RG_TR)>(p, tile); break;
+    case RG_T: tile_body<Op, MODE, region_checks(RG_T)>(p, tile); break;
+    case RG_BL: tile_body<Op, MODE, region_checks(RG_BL)>(p, tile); break;
+    case RG_BR: tile_body<Op, MODE, region_checks(RG_BR)>(p, tile); break;
+    case RG_B: tile_body<Op, MODE, region_checks(RG_B)>(p, tile); break;
+    case RG_R: tile_body<Op, MODE, region_checks(RG_R)>(p, tile); break;
+    case RG_L: tile_body<Op, MODE, region_checks(RG_L)>(p, tile); break;
+    default: tile_body<Op, MODE, 0>(p, tile); break;
+    }
+}
+
+// Strided store of the tiled form: element e is column x + 32 e (guarded in R regions).
+template <int CK, class T, int PX>
+__device__ __forceinline__ void store_strided_px(T *__restrict__ row, int x, int w, const T (&v)[PX])
+{
+#pragma unroll
+    for (int e = 0; e < PX; ++e)
+        if (!(CK & CK_R) || x + 32 * e < w) row[x + 32 * e] = v[e];
+}
+
 // Generic f32 local operator with a runtime window (<= 31 x 31).  Same FMA order as
 // OpConvF32 (row-major taps), so both families give identical bits.
 struct DOpConvF32 {
     using Tin = float;
     static constexpr int PX = 4, MAXT = 31 * 31;
+    static constexpr bool TILED = true;
     struct Params {
         Geom g;
         const float *in;
@@ -118,12 +215,19 @@ struct DOpConvF32 {
     {
         store_px<CK, float, PX>(p.out + (ptrdiff_t)(y - p.g.oy0) * p.g.out_pitch, x0, p.g.w, p.g.vec_out, a.v);
     }
+    __device__ __forceinline__ static void init_tile(const Params &p, A &a, const float *) { init(p, a, 0, 0); }
+    template <int CK>
+    __device__ __forceinline__ static void store_strided(const Params &p, const A &a, int x, int y)
+    {
+        store_strided_px<CK, float, PX>(p.out + (ptrdiff_t)(y - p.g.oy0) * p.g.out_pitch, x, p.g.w, a.v);
+    }
 };
 
 // Generic u8 local operator, runtime window, int32 mask.
 struct DOpConvU8 {
     using Tin = uint8_t;
     static constexpr int PX = 4, MAXT = 31 * 31;
+    static constexpr bool TILED = false;
     struct Params {
         Geom g;
         const uint8_t *in;
@@ -168,6 +272,7 @@ __device__ __forceinline__ float ex2_approx(float x)
 struct DOpBilateral {
     using Tin = float;
     static constexpr int PX = 4, MAXT = 31 * 31;
+    static constexpr bool TILED = true;
     struct Params {
         Geom g;
         const float *in;
@@ -188,15 +293,33 @@ struct DOpBilateral {
             a.den[e] = 0.f;
         }
     }
+    // per output: d = I_q - I_p, w = 2^(d*d*kr + ls), num += w I_q, den += w -- two outputs
+    // per instruction with the sm_100 packed FP32 ops (each lane an IEEE op: the same
+    // bits as the scalar sequence)
     __device__ __forceinline__ static void tap(const Params &p, int j, int i, const float (&win)[PX], A &a)
     {
         const float ls = p.ls[j * p.mw + i];
+        unsigned long long kr2, ls2;
+        asm("mov.b64 %0, {%1, %1};" : "=l"(kr2) : "f"(p.kr));
+        asm("mov.b64 %0, {%1, %1};" : "=l"(ls2) : "f"(ls));
 #pragma unroll
-        for (int e = 0; e < PX; ++e) {
-            const float d = win[e] - a.c[e];
-            const float wgt = ex2_approx(fmaf(d * d, p.kr, ls));
-            a.num[e] = fmaf(wgt, win[e], a.num[e]);
-            a.den[e] += wgt;
+        for (int e = 0; e < PX; e += 2) {
+            unsigned long long wv, nc, d, t, num, den, wg;
+            asm("mov.b64 %0, {%1, %2};" : "=l"(wv) : "f"(win[e]), "f"(win[e + 1]));
+            asm("mov.b64 %0, {%1, %2};" : "=l"(nc) : "f"(-a.c[e]), "f"(-a.c[e + 1]));
+            asm("add.rn.f32x2 %0, %1, %2;" : "=l"(d) : "l"(wv), "l"(nc));
+            asm("mul.rn.f32x2 %0, %1, %1;" : "=l"(t) : "l"(d));
+            asm("fma.rn.f32x2 %0, %1, %2, %3;" : "=l"(t) : "l"(t), "l"(kr2), "l"(ls2));
+            float t0, t1;
+            asm("mov.b64 {%0, %1}, %2;" : "=f"(t0), "=f"(t1) : "l"(t));
+            const float w0 = ex2_approx(t0), w1 = ex2_approx(t1);
+            asm("mov.b64 %0, {%1, %2};" : "=l"(wg) : "f"(w0), "f"(w1));
+            asm("mov.b64 %0, {%1, %2};" : "=l"(num) : "f"(a.num[e]), "f"(a.num[e + 1]));
+            asm("mov.b64 %0, {%1, %2};" : "=l"(den) : "f"(a.den[e]), "f"(a.den[e + 1]));
+            asm("fma.rn.f32x2 %0, %1, %2, %0;" : "+l"(num) : "l"(wg), "l"(wv));
+            asm("add.rn.f32x2 %0, %0, %1;" : "+l"(den) : "l"(wg));
+            asm("mov.b64 {%0, %1}, %2;" : "=f"(a.num[e]), "=f"(a.num[e + 1]) : "l"(num));
+            asm("mov.b64 {%0, %1}, %2;" : "=f"(a.den[e]), "=f"(a.den[e + 1]) : "l"(den));
         }
     }
     template <int CK>
@@ -206,6 +329,24 @@ struct DOpBilateral {
 #pragma unroll
         for (int e = 0; e < PX; ++e) o[e] = a.num[e] / a.den[e];
         store_px<CK, float, PX>(p.out + (ptrdiff_t)(y - p.g.oy0) * p.g.out_pitch, x0, p.g.w, p.g.vec_out, o);
+    }
+    // tiled form: centre values from the smem tile (element e at column +32 e)
+    __device__ __forceinline__ static void init_tile(const Params &, A &a, const float *ctr)
+    {
+#pragma unroll
+        for (int e = 0; e < PX; ++e) {
+            a.c[e] = ctr[32 * e];
+            a.num[e] = 0.f;
+            a.den[e] = 0.f;
+        }
+    }
+    template <int CK>
+    __device__ __forceinline__ static void store_strided(const Params &p, const A &a, int x, int y)
+    {
+        float o[PX];
+#pragma unroll
+        for (int e = 0; e < PX; ++e) o[e] = a.num[e] / a.den[e];
+        store_strided_px<CK, float, PX>(p.out + (ptrdiff_t)(y - p.g.oy0) * p.g.out_pitch, x, p.g.w, o);
     }
 };
 

@@ -19,6 +19,9 @@ const void *kernel_for_disp(int disp)
         case DISP_BLOCK: return (const void *)k_direct<Op, MODE, DISP_BLOCK>;
         case DISP_WARP: return (const void *)k_direct<Op, MODE, DISP_BLOCK>;
         case DISP_NAIVE: return (const void *)k_direct<Op, MODE, DISP_NAIVE>;
+        case DISP_TMA:
+            if constexpr (Op::TILED) return (const void *)k_tile<Op, MODE>;
+            else return nullptr;
         default:
             if constexpr (MODE == MIRROR) return (const void *)k_direct<Op, MODE, DISP_NAIVE_GEN>;
             else return (const void *)k_direct<Op, MODE, DISP_NAIVE>;

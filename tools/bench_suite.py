@@ -165,7 +165,7 @@ def cfg4(sweep=True):
         return rec(us, n * n, 8 * n * n, plan, {"ex2_per_s": nexp / (us * 1e-6),
                                                 "mufu_frac": nexp / (us * 1e-6) / mufu_peak})
 
-    res = {"win13": {m: {v: one(13, m, v) for v in ["auto", "warp", "naive"]} for m in MODES}}
+    res = {"win13": {m: {v: one(13, m, v) for v in ["auto", "tma", "warp", "naive"]} for m in MODES}}
     if sweep:
         sw = {}
         for m in MODES:
@@ -174,7 +174,9 @@ def cfg4(sweep=True):
                 a = one(win, m, "auto")
                 w = one(win, m, "warp")
                 nv = one(win, m, "naive")
+                t = one(win, m, "tma")
                 rows.append({"win": win, "isp_us": w["us"], "naive_us": nv["us"], "speedup": nv["us"] / w["us"],
+                             "tiled_us": t["us"], "tiled_mufu_frac": t["mufu_frac"], "auto_us": a["us"],
                              "G": a["G"], "auto_choice": a["choice"]})
             sp = np.array([r["speedup"] for r in rows])
             G = np.array([r["G"] for r in rows])
