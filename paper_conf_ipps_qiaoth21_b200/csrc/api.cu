@@ -254,7 +254,9 @@ int family_px(int fam, bool direct)
 {
     if (direct) return PX_DIRECT;
     switch (fam) {
-    case F_U8: case F_SOBEL: case F_LAPLACE: return PX_U8;
+    case F_U8: return PX_U8;
+    case F_SOBEL: return kPxSobel;
+    case F_LAPLACE: return kPxLaplace;
     case F_HARRIS: return PX_I16;
     default: return PX_F32;
     }

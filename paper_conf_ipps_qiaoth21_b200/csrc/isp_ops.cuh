@@ -161,7 +161,7 @@ template <int MW_, int MH_>
 struct OpConvU8 {
     using Tin = uint8_t;
     static constexpr int NIN = 1, PX = kPxU8, HX = MW_ / 2, HY = MH_ / 2, MH = MH_, SEGW = PX + 2 * HX;
-    static constexpr int PFMAX = 0;
+    static constexpr int PFMAX = kPfSub;  // rows loaded ahead (latency hiding)
     static constexpr bool ROW_DIRECT = false;
     static constexpr bool SHFL_HALO = false;  // shuffle halo measured slower
     struct Params {
@@ -210,7 +210,7 @@ template <int MW_, int MH_>
 struct OpSepU8 {
     using Tin = uint8_t;
     static constexpr int NIN = 1, PX = kPxU8, HX = MW_ / 2, HY = MH_ / 2, MH = MH_, SEGW = PX + 2 * HX;
-    static constexpr int PFMAX = 0;
+    static constexpr int PFMAX = kPfSub;  // rows loaded ahead (latency hiding)
     static constexpr bool ROW_DIRECT = false;
     static constexpr bool SHFL_HALO = false;  // shuffle halo measured slower
     struct Params {
@@ -276,8 +276,8 @@ __device__ __forceinline__ int sobel_mag(int n)
 // ---------------------------------------------------------------------------------
 struct OpSobel {
     using Tin = uint8_t;
-    static constexpr int NIN = 1, PX = kPxU8, HX = 1, HY = 1, MH = 3, SEGW = PX + 2;
-    static constexpr int PFMAX = 0;
+    static constexpr int NIN = 1, PX = kPxSobel, HX = 1, HY = 1, MH = 3, SEGW = PX + 2;
+    static constexpr int PFMAX = kPfSub;  // rows loaded ahead (latency hiding)
     static constexpr bool ROW_DIRECT = false;
     static constexpr bool SHFL_HALO = false;  // shuffle halo measured slower
     struct Params {
@@ -342,10 +342,12 @@ struct OpSobel {
 };
 
 // Laplace 5x5 (a8): box sum minus 25 x centre (== ones mask with centre -24).
+// One accumulator per output (the centre term enters with the centre row, j == 2), and
+// the horizontal 5-sums slide (2 ops per pixel after the first).
 struct OpLaplace5 {
     using Tin = uint8_t;
-    static constexpr int NIN = 1, PX = kPxU8, HX = 2, HY = 2, MH = 5, SEGW = PX + 4;
-    static constexpr int PFMAX = 0;
+    static constexpr int NIN = 1, PX = kPxLaplace, HX = 2, HY = 2, MH = 5, SEGW = PX + 4;
+    static constexpr int PFMAX = kPfSub;  // rows loaded ahead (latency hiding)
     static constexpr bool ROW_DIRECT = false;
     static constexpr bool SHFL_HALO = false;  // shuffle halo measured slower
     struct Params {
@@ -355,40 +357,41 @@ struct OpLaplace5 {
         uint8_t *out;
     };
     struct H { int box[PX], ctr[PX]; };
-    using A = AccI<PX, 2>;
+    using A = AccI<PX, 1>;
     __host__ __device__ static constexpr bool col_used(int) { return true; }
     __host__ __device__ static constexpr bool row_used(int) { return true; }
     __device__ __forceinline__ static void zero(A &a)
     {
 #pragma unroll
-        for (int e = 0; e < PX; ++e) a.v[0][e] = a.v[1][e] = 0;
+        for (int e = 0; e < PX; ++e) a.v[0][e] = 0;
     }
     __device__ __forceinline__ static void hrow(const Params &, const uint8_t (&seg)[1][SEGW], H &h)
     {
+        int s = 0;
 #pragma unroll
-        for (int e = 0; e < PX; ++e) {
-            int s = 0;
+        for (int i = 0; i < 5; ++i) s += seg[0][i];
+        h.box[0] = s;
 #pragma unroll
-            for (int i = 0; i < 5; ++i) s += seg[0][e + i];
+        for (int e = 1; e < PX; ++e) {
+            s += (int)seg[0][e + 4] - (int)seg[0][e - 1];
             h.box[e] = s;
-            h.ctr[e] = seg[0][e + 2];
         }
+#pragma unroll
+        for (int e = 0; e < PX; ++e) h.ctr[e] = seg[0][e + 2];
     }
     template <bool FIRST>
     __device__ __forceinline__ static void vacc(const Params &, int j, const H &h, A &a)
     {
 #pragma unroll
-        for (int e = 0; e < PX; ++e) {
-            a.v[0][e] = (FIRST ? 0 : a.v[0][e]) + h.box[e];
-            if (j == 2) a.v[1][e] = h.ctr[e];
-        }
+        for (int e = 0; e < PX; ++e)
+            a.v[0][e] = (FIRST ? 0 : a.v[0][e]) + (j == 2 ? h.box[e] - 25 * h.ctr[e] : h.box[e]);
     }
     template <int CK>
     __device__ __forceinline__ static void store(const Params &p, const A &a, int x0, int y)
     {
         uint8_t o[PX];
 #pragma unroll
-        for (int e = 0; e < PX; ++e) o[e] = sat_u8(a.v[0][e] - 25 * a.v[1][e]);
+        for (int e = 0; e < PX; ++e) o[e] = sat_u8(a.v[0][e]);
         store_px<CK, uint8_t, PX>(p.out + (ptrdiff_t)(y - p.g.oy0) * p.g.out_pitch, x0, p.g.w, p.g.vec_out, o);
     }
 };
@@ -398,7 +401,7 @@ struct OpLaplace5 {
 struct OpHarris {
     using Tin = int16_t;
     static constexpr int NIN = 2, PX = 4, HX = 1, HY = 1, MH = 3, SEGW = PX + 2;
-    static constexpr int PFMAX = 0;
+    static constexpr int PFMAX = kPfSub;  // rows loaded ahead (latency hiding)
     static constexpr bool ROW_DIRECT = false;
     static constexpr bool SHFL_HALO = false;  // shuffle halo measured slower
     struct Params {

@@ -146,6 +146,38 @@ __device__ __forceinline__ typename Op::Tin fixup_value(const typename Op::Tin *
     }
 }
 
+// Clamp and Mirror columns beyond a side are copies of columns inside the tile, so
+// when the width is a whole number of vectors (no partial vector at the right edge) the
+// compute warps rebuild them in registers (staged_edge_fix) and the producer issues no
+// column fix-ups at all: L/R CTAs then stage exactly like Body CTAs.
+__device__ __forceinline__ bool consumer_fix(const Geom &g, int px)
+{
+    return (g.mode == CLAMP || g.mode == MIRROR) && g.w % px == 0 && g.w_al == g.w && g.dbg != 5;
+}
+
+template <class Op, int CK>
+__device__ __forceinline__ void staged_edge_fix(const Geom &g, int x0, typename Op::Tin (&seg)[Op::NIN][Op::PX + 2 * Op::HX])
+{
+    constexpr int PX = Op::PX, HX = Op::HX;
+    const bool mirror = g.mode == MIRROR;
+#pragma unroll
+    for (int c = 0; c < Op::NIN; ++c) {
+        if constexpr ((CK & CK_L) != 0) {
+            if (x0 == 0) {  // columns -HX..-1 <- 0 (Clamp) / HX-1..0 (Mirror)
+#pragma unroll
+                for (int k = 0; k < HX; ++k) seg[c][k] = mirror ? seg[c][2 * HX - 1 - k] : seg[c][HX];
+            }
+        }
+        if constexpr ((CK & CK_R) != 0) {
+            if (x0 + PX == g.w) {  // columns w..w+HX-1 <- w-1 (Clamp) / w-1..w-HX (Mirror)
+#pragma unroll
+                for (int t = 0; t < HX; ++t)
+                    seg[c][HX + PX + t] = mirror ? seg[c][HX + PX - 1 - t] : seg[c][HX + PX - 1];
+            }
+        }
+    }
+}
+
 // Producer warp of a staged CTA (the only mode-dependent code: row maps, fix-ups).
 template <class Op, int MODE, int CK>
 __device__ __forceinline__ void staged_producer(const typename Op::Params &p, uint64_t *full, uint64_t *empty,
@@ -190,7 +222,7 @@ __device__ __forceinline__ void staged_producer(const typename Op::Params &p, ui
                 for (int c = 0; c < NIN; ++c)
                     bulk_g2s(rb + (size_t)c * SW + (cs - XS), p.in[c] + (ptrdiff_t)yy * g.in_pitch + cs,
                              (uint32_t)(ce - cs) * (uint32_t)sizeof(T), &full[s]);
-            if (CK != 0 && g.dbg != 4) {
+            if (CK != 0 && g.dbg != 4 && !((CK & (CK_L | CK_R)) && consumer_fix(g, PX))) {
                 // border fix-ups, this region's sides only (<= HXA columns per row):
                 // cp.async of the pattern's source column (4-byte types), else a
                 // synchronous copy; Constant: the constant
@@ -220,7 +252,7 @@ __device__ __forceinline__ void staged_producer(const typename Op::Params &p, ui
             }
         }
         if constexpr (ASYNC_FIX) {
-            if (g.dbg != 4) cp_async_mbar_arrive_noinc(&full[s]);
+            if (g.dbg != 4 && !consumer_fix(g, PX)) cp_async_mbar_arrive_noinc(&full[s]);
         }
         if constexpr (MODE == CONSTANT && (CK & (CK_T | CK_B)) != 0)
             fence_proxy_async();  // generic row fills before later bulk (async-proxy) writes
@@ -255,7 +287,7 @@ __device__ __forceinline__ void staged_body(const typename Op::Params &p, unsign
     const bool async_fix = (CK & (CK_L | CK_R)) != 0 && sizeof(T) == 4 && g.mode != CONSTANT;
     if (threadIdx.x == 0) {
         for (int s = 0; s < S; ++s) {
-            mbar_init(&full[s], async_fix && g.dbg != 4 ? 33 : 1);
+            mbar_init(&full[s], async_fix && g.dbg != 4 && !consumer_fix(g, Op::PX) ? 33 : 1);
             mbar_init(&empty[s], NWC);
         }
         fence_mbar_init();
@@ -305,6 +337,9 @@ __device__ __forceinline__ void staged_body(const typename Op::Params &p, unsign
                 if (g.dbg == 1) continue;
                 T seg[NIN][SEGW];
                 unpack_row<Op>(rr, seg);
+                if constexpr ((CK & (CK_L | CK_R)) != 0) {
+                    if (consumer_fix(g, PX)) staged_edge_fix<Op, CK>(g, x0, seg);
+                }
                 typename Op::H hs;
                 Op::hrow(p, seg, hs);
                 // every tap unconditionally: j == 0 initialises the row's accumulator, so
