@@ -397,7 +397,19 @@ struct OpLaplace5 {
 };
 
 // Harris over (dx, dy) int16 (a10; BASELINE configs[2]): 3x3, w = [1,2,1](x)[1,2,1].
-// Sxx, Syy, Sxy < 2^25 fit int32 exactly; R25 in int64.
+// Exact in floating point: |dx|, |dy| <= 1020, so every product (<= 1020^2) and every
+// weighted sum Sxx, Syy, |Sxy| <= 16 * 1020^2 = 16,646,400 < 2^24 is an integer that f32
+// represents exactly, in any summation order.  The response
+// R25 = 25 (Sxx Syy - Sxy^2) - (Sxx + Syy)^2 has every intermediate below 2^53 in
+// magnitude (25 * Sxx * Syy <= 6.9e15), so f64 evaluates it exactly; the comparison with
+// the int64 threshold is exact after clamping it to +-2^53.  Same bits as the int64
+// definition (oracle) by construction.
+__device__ __forceinline__ float i16_to_f32(int x)
+{
+    // 1.5 * 2^23 + x has the integer x in its low mantissa bits for |x| < 2^22
+    return __int_as_float(0x4B400000 + x) - 12582912.0f;
+}
+
 struct OpHarris {
     using Tin = int16_t;
     static constexpr int NIN = 2, PX = 4, HX = 1, HY = 1, MH = 3, SEGW = PX + 2;
@@ -411,53 +423,65 @@ struct OpHarris {
         long long thr;
         uint8_t *out;
     };
-    struct H { int xx[PX], yy[PX], xy[PX]; };
-    using A = AccI<PX, 3>;
+    struct H { float xx[PX], yy[PX], xy[PX]; };
+    struct A { float v[3][PX]; };
     __host__ __device__ static constexpr bool col_used(int) { return true; }
     __host__ __device__ static constexpr bool row_used(int) { return true; }
     __device__ __forceinline__ static void zero(A &a)
     {
 #pragma unroll
-        for (int e = 0; e < PX; ++e) a.v[0][e] = a.v[1][e] = a.v[2][e] = 0;
+        for (int e = 0; e < PX; ++e) a.v[0][e] = a.v[1][e] = a.v[2][e] = 0.f;
     }
     __device__ __forceinline__ static void hrow(const Params &, const int16_t (&seg)[2][SEGW], H &h)
     {
-        int pxx[SEGW], pyy[SEGW], pxy[SEGW];
+        float pxx[SEGW], pyy[SEGW], pxy[SEGW];
 #pragma unroll
-        for (int k = 0; k < SEGW; ++k) {
-            const int gx = seg[0][k], gy = seg[1][k];
-            pxx[k] = gx * gx;
-            pyy[k] = gy * gy;
-            pxy[k] = gx * gy;
+        for (int k = 0; k < SEGW; k += 2) {
+            const float gx0 = i16_to_f32(seg[0][k]), gx1 = i16_to_f32(seg[0][k + 1]);
+            const float gy0 = i16_to_f32(seg[1][k]), gy1 = i16_to_f32(seg[1][k + 1]);
+            pxx[k] = gx0 * gx0;
+            pxx[k + 1] = gx1 * gx1;
+            pyy[k] = gy0 * gy0;
+            pyy[k + 1] = gy1 * gy1;
+            pxy[k] = gx0 * gy0;
+            pxy[k + 1] = gx1 * gy1;
         }
 #pragma unroll
         for (int e = 0; e < PX; ++e) {
-            h.xx[e] = pxx[e] + 2 * pxx[e + 1] + pxx[e + 2];
-            h.yy[e] = pyy[e] + 2 * pyy[e + 1] + pyy[e + 2];
-            h.xy[e] = pxy[e] + 2 * pxy[e + 1] + pxy[e + 2];
+            h.xx[e] = fmaf(2.f, pxx[e + 1], pxx[e]) + pxx[e + 2];
+            h.yy[e] = fmaf(2.f, pyy[e + 1], pyy[e]) + pyy[e + 2];
+            h.xy[e] = fmaf(2.f, pxy[e + 1], pxy[e]) + pxy[e + 2];
         }
     }
     template <bool FIRST>
     __device__ __forceinline__ static void vacc(const Params &, int j, const H &h, A &a)
     {
-        const int wj = (j == 1) ? 2 : 1;
+        const float wj = (j == 1) ? 2.f : 1.f;
 #pragma unroll
-        for (int e = 0; e < PX; ++e) {
-            a.v[0][e] = (FIRST ? 0 : a.v[0][e]) + wj * h.xx[e];
-            a.v[1][e] = (FIRST ? 0 : a.v[1][e]) + wj * h.yy[e];
-            a.v[2][e] = (FIRST ? 0 : a.v[2][e]) + wj * h.xy[e];
+        for (int e = 0; e < PX; e += 2) {
+            if (FIRST) {
+                a.v[0][e] = h.xx[e]; a.v[0][e + 1] = h.xx[e + 1];
+                a.v[1][e] = h.yy[e]; a.v[1][e + 1] = h.yy[e + 1];
+                a.v[2][e] = h.xy[e]; a.v[2][e + 1] = h.xy[e + 1];
+            } else {
+                fma2(a.v[0][e], a.v[0][e + 1], wj, h.xx[e], h.xx[e + 1]);
+                fma2(a.v[1][e], a.v[1][e + 1], wj, h.yy[e], h.yy[e + 1]);
+                fma2(a.v[2][e], a.v[2][e + 1], wj, h.xy[e], h.xy[e + 1]);
+            }
         }
     }
     template <int CK>
     __device__ __forceinline__ static void store(const Params &p, const A &a, int x0, int y)
     {
+        const double thr = (double)max(-9007199254740992ll, min(9007199254740992ll, p.thr));  // +-2^53
         uint8_t o[PX];
 #pragma unroll
         for (int e = 0; e < PX; ++e) {
-            const long long sxx = a.v[0][e], syy = a.v[1][e], sxy = a.v[2][e];
-            const long long tr = sxx + syy;
-            const long long r25 = 25 * (sxx * syy - sxy * sxy) - tr * tr;
-            o[e] = r25 > p.thr ? 255 : 0;
+            const double sxx = a.v[0][e], syy = a.v[1][e], sxy = a.v[2][e];
+            const double det = fma(-sxy, sxy, sxx * syy);      // exact: all terms < 2^49
+            const double tr = sxx + syy;                        // exact
+            const double r25 = fma(25.0, det, -(tr * tr));      // exact: |.| < 2^53
+            o[e] = r25 > thr ? 255 : 0;
         }
         store_px<CK, uint8_t, PX>(p.out + (ptrdiff_t)(y - p.g.oy0) * p.g.out_pitch, x0, p.g.w, p.g.vec_out, o);
     }
