@@ -391,6 +391,9 @@ isp_status_t resolve_and_launch(Desc &d, int fam, int w, int h, int mw, int mh, 
         return make_plan(w, h, hx, hy, px, 0, g_override_ty > 0 ? 0 : ty, 0, rr,
                          c == ISP_NAIVE ? nb_naive : nb_stream);
     };
+    // the streaming ISP bodies assume vector-aligned rows (isp_core.cuh load_row):
+    // misaligned images run the naive kernel (identical results)
+    if (!direct && !d.g.vec_in && (chosen == ISP_BLOCK || chosen == ISP_WARP)) chosen = ISP_NAIVE;
     Plan p = plan_for(chosen);
     isp_plan_info info{};
     if (p.degenerate) chosen = ISP_NAIVE;  // A3: Listing 3 cannot express a block needing opposite checks
