@@ -412,7 +412,7 @@ __device__ __forceinline__ float i16_to_f32(int x)
 
 struct OpHarris {
     using Tin = int16_t;
-    static constexpr int NIN = 2, PX = 4, HX = 1, HY = 1, MH = 3, SEGW = PX + 2;
+    static constexpr int NIN = 2, PX = kPxI16, HX = 1, HY = 1, MH = 3, SEGW = PX + 2;
     static constexpr int PFMAX = kPfSub;  // rows loaded ahead (latency hiding)
     static constexpr bool ROW_DIRECT = false;
     static constexpr bool SHFL_HALO = false;  // shuffle halo measured slower

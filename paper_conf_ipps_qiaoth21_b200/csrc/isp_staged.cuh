@@ -146,33 +146,35 @@ __device__ __forceinline__ typename Op::Tin fixup_value(const typename Op::Tin *
     }
 }
 
-// Clamp and Mirror columns beyond a side are copies of columns inside the tile, so
+// Clamp and Mirror columns beyond a side are copies of columns inside the tile (and
+// Constant columns are C), so
 // when the width is a whole number of vectors (no partial vector at the right edge) the
 // compute warps rebuild them in registers (staged_edge_fix) and the producer issues no
 // column fix-ups at all: L/R CTAs then stage exactly like Body CTAs.
 __device__ __forceinline__ bool consumer_fix(const Geom &g, int px)
 {
-    return (g.mode == CLAMP || g.mode == MIRROR) && g.w % px == 0 && g.w_al == g.w && g.dbg != 5;
+    return g.mode != REPEAT && g.w % px == 0 && g.w_al == g.w && g.dbg != 5;
 }
 
 template <class Op, int CK>
-__device__ __forceinline__ void staged_edge_fix(const Geom &g, int x0, typename Op::Tin (&seg)[Op::NIN][Op::PX + 2 * Op::HX])
+__device__ __forceinline__ void staged_edge_fix(const Geom &g, int x0, typename Op::Tin (&seg)[Op::NIN][Op::PX + 2 * Op::HX],
+                                                typename Op::Tin cval)
 {
     constexpr int PX = Op::PX, HX = Op::HX;
-    const bool mirror = g.mode == MIRROR;
+    const bool mirror = g.mode == MIRROR, cst = g.mode == CONSTANT;
 #pragma unroll
     for (int c = 0; c < Op::NIN; ++c) {
         if constexpr ((CK & CK_L) != 0) {
             if (x0 == 0) {  // columns -HX..-1 <- 0 (Clamp) / HX-1..0 (Mirror)
 #pragma unroll
-                for (int k = 0; k < HX; ++k) seg[c][k] = mirror ? seg[c][2 * HX - 1 - k] : seg[c][HX];
+                for (int k = 0; k < HX; ++k) seg[c][k] = cst ? cval : mirror ? seg[c][2 * HX - 1 - k] : seg[c][HX];
             }
         }
         if constexpr ((CK & CK_R) != 0) {
             if (x0 + PX == g.w) {  // columns w..w+HX-1 <- w-1 (Clamp) / w-1..w-HX (Mirror)
 #pragma unroll
                 for (int t = 0; t < HX; ++t)
-                    seg[c][HX + PX + t] = mirror ? seg[c][HX + PX - 1 - t] : seg[c][HX + PX - 1];
+                    seg[c][HX + PX + t] = cst ? cval : mirror ? seg[c][HX + PX - 1 - t] : seg[c][HX + PX - 1];
             }
         }
     }
@@ -222,7 +224,9 @@ __device__ __forceinline__ void staged_producer(const typename Op::Params &p, ui
                 for (int c = 0; c < NIN; ++c)
                     bulk_g2s(rb + (size_t)c * SW + (cs - XS), p.in[c] + (ptrdiff_t)yy * g.in_pitch + cs,
                              (uint32_t)(ce - cs) * (uint32_t)sizeof(T), &full[s]);
-            if (CK != 0 && g.dbg != 4 && !((CK & (CK_L | CK_R)) && consumer_fix(g, PX))) {
+            if (CK != 0 && g.dbg != 4) {
+                // column fix-ups unless the compute warps rebuild the edge columns
+                const bool colfix = !((CK & (CK_L | CK_R)) && consumer_fix(g, PX));
                 // border fix-ups, this region's sides only (<= HXA columns per row):
                 // cp.async of the pattern's source column (4-byte types), else a
                 // synchronous copy; Constant: the constant
@@ -233,6 +237,7 @@ __device__ __forceinline__ void staged_producer(const typename Op::Params &p, ui
                         for (int x = lane; x < SW; x += 32) dst[x] = p.cval;
                         continue;
                     }
+                    if (!colfix) continue;
                     const T *src = p.in[c] + (ptrdiff_t)yy * g.in_pitch;
                     auto fix = [&](int x) {
                         if constexpr (MODE == CONSTANT) {
@@ -338,7 +343,7 @@ __device__ __forceinline__ void staged_body(const typename Op::Params &p, unsign
                 T seg[NIN][SEGW];
                 unpack_row<Op>(rr, seg);
                 if constexpr ((CK & (CK_L | CK_R)) != 0) {
-                    if (consumer_fix(g, PX)) staged_edge_fix<Op, CK>(g, x0, seg);
+                    if (consumer_fix(g, PX)) staged_edge_fix<Op, CK>(g, x0, seg, p.cval);
                 }
                 typename Op::H hs;
                 Op::hrow(p, seg, hs);
