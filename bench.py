@@ -167,7 +167,7 @@ def run_reference(args):
     img = synth.uniform_f32(N_SIDE, N_SIDE, synth.CONFIG_SEEDS["cfg2"])
     mask = gauss_mask()
     # each step = a bounded sample (rows_per_step rows x 4 modes), sized so the run ends in minutes
-    rows_per_step = max(threads, 8 * threads // 8)
+    rows_per_step = 16 * threads  # 16 rows per host thread and mode: amortises the per-call setup
     times = []
     for k in range(args.warmup + args.steps):
         y0 = (k * rows_per_step) % (N_SIDE - rows_per_step)
