@@ -114,6 +114,22 @@ isp_status_t isp_harris_u8(const int16_t *dx, const int16_t *dy, int w, int h, i
                            int const_val, int64_t thr, uint8_t *out, int out_pitch, isp_variant_t variant,
                            isp_stream_t stream);
 
+/* BASELINE.json configs[2] fused into ONE launch (Sobel, Laplace from
+ * P:L355, Harris a10): reads the u8 image once and writes mag, lap, harris (u8) and,
+ * if non-NULL, dx and dy (int16).  Bit-identical to
+ *   isp_sobel_u8(img, mode, const_val) -> dx, dy, mag;  isp_laplace5_u8(img, mode, const_val);
+ *   isp_harris_u8(dx, dy, mode, harris_const, thr)
+ * i.e. Harris' border handling applies to the dx/dy IMAGES (remapped coordinates).
+ * All outputs share out_pitch (elements); img is caller-owned device memory, pitch in
+ * bytes = elements.  ISP_NAIVE stages every tile through the checked gather; any other
+ * variant runs Body tiles unchecked.  EINVAL: sizes/pitches, mode, NULL mag/lap/harris,
+ * const_val not in [0,255], harris_const not in [-1020,1020] (the Sobel range; keeps the
+ * int32 window sums exact).  EALIAS: an output overlaps img.  Stream-ordered. */
+isp_status_t isp_pipeline_cfg3_u8(const uint8_t *img, int w, int h, int pitch, int border_mode, int const_val,
+                                  int harris_const, int64_t thr, int16_t *dx, int16_t *dy, uint8_t *mag,
+                                  uint8_t *lap, uint8_t *harris, int out_pitch, isp_variant_t variant,
+                                  isp_stream_t stream);
+
 /* Bilateral filter (a11), f32, window win x win (odd, <= 31):
  *   out(p) = sum_q s(q-p) r(I_q-I_p) I_q / sum_q s(q-p) r(I_q-I_p),
  *   s = exp(-(dx^2+dy^2)/(2 sigma_d^2)), r(d) = exp(-d^2/(2 sigma_r^2)).

@@ -23,7 +23,7 @@ __all__ = [
     "CLAMP", "MIRROR", "REPEAT", "CONSTANT", "AUTO", "BLOCK", "WARP", "NAIVE", "TMA", "MODES", "VARIANTS",
     "lib", "IspError", "PlanInfo", "ModelParams",
     "isp_filter", "isp_filter_naive", "isp_filter_ex", "isp_filter_sep_f32", "isp_filter_u8",
-    "isp_sobel_u8", "isp_laplace5_u8", "isp_harris_u8", "isp_bilateral_f32", "isp_atrous_f32",
+    "isp_sobel_u8", "isp_laplace5_u8", "isp_harris_u8", "isp_pipeline_cfg3_u8", "isp_bilateral_f32", "isp_atrous_f32",
     "isp_night_f32", "isp_plan", "isp_model_defaults", "isp_last_plan", "isp_set_launch_override",
     "isp_shard_unique_id", "isp_shard_init", "isp_shard_rows", "isp_shard_schedule",
     "isp_shard_filter_f32", "isp_shard_filter_u8", "isp_shard_filter_local_f32", "isp_shard_destroy",
@@ -95,6 +95,7 @@ _SIGS = {
     "isp_sobel_u8": [_P, _I, _I, _I, _I, _I, _P, _P, _P, _I, _I, _P],
     "isp_laplace5_u8": [_P, _I, _I, _I, _I, _I, _P, _I, _I, _P],
     "isp_harris_u8": [_P, _P, _I, _I, _I, _I, _I, ctypes.c_int64, _P, _I, _I, _P],
+    "isp_pipeline_cfg3_u8": [_P, _I, _I, _I, _I, _I, _I, ctypes.c_int64, _P, _P, _P, _P, _P, _I, _I, _P],
     "isp_bilateral_f32": [_P, _I, _I, _I, _I, _F, _F, _I, _F, _P, _I, _I, _P],
     "isp_atrous_f32": [_P, _I, _I, _I, _I, _I, _F, _I, _P, _I, _I, _P],
     "isp_night_f32": [_P, _I, _I, _I, _I, _F, _P, _P, _P, _I, _I, _P],
@@ -266,6 +267,28 @@ def isp_harris_u8(dx, dy, border_mode, const_val=0, thr=0, out=None, variant=AUT
     _check(lib().isp_harris_u8(dx.data_ptr(), dy.data_ptr(), w, h, pitch, _mode(border_mode), int(const_val),
                                int(thr), out.data_ptr(), out.shape[1], _variant(variant), _stream(dx, stream)))
     return out
+
+
+def isp_pipeline_cfg3_u8(img, border_mode, const_val=0, harris_const=0, thr=0, mag=None, lap=None, harris=None,
+                         dx=None, dy=None, variant=AUTO, w=None, stream=None):
+    """Sobel + Laplace 5x5 + Harris in one launch (include/isp.h); dx/dy written only if given.
+    Returns (mag, lap, harris)."""
+    _img(img, torch.uint8)
+    w, h, pitch = _geom(img, w)
+    mag = _out(mag, img, w, torch.uint8)
+    lap = _out(lap, img, w, torch.uint8)
+    harris = _out(harris, img, w, torch.uint8)
+    op = mag.shape[1]
+    for t, dt in ((lap, torch.uint8), (harris, torch.uint8), (dx, torch.int16), (dy, torch.int16)):
+        if t is not None:
+            _img(t, dt, "out")
+            if t.shape[1] != op:
+                raise ValueError("all outputs must share out_pitch")
+    ptr = lambda t: t.data_ptr() if t is not None else None  # noqa: E731
+    _check(lib().isp_pipeline_cfg3_u8(img.data_ptr(), w, h, pitch, _mode(border_mode), int(const_val),
+                                      int(harris_const), int(thr), ptr(dx), ptr(dy), mag.data_ptr(), lap.data_ptr(),
+                                      harris.data_ptr(), op, _variant(variant), _stream(img, stream)))
+    return mag, lap, harris
 
 
 def isp_bilateral_f32(img, win, sigma_d, sigma_r, border_mode, const_val=0.0, out=None, variant=AUTO, w=None,

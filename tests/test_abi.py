@@ -126,3 +126,19 @@ def test_shard_schedule(mode, Pn):
     assert sends.keys() == recvs.keys()
     for key in sends:
         assert [n for _, n in sends[key]] == [n for _, n in recvs[key]]
+
+
+def test_pipeline_cfg3_validation():
+    """isp_pipeline_cfg3_u8 argument checks (include/isp.h) fail before any device work."""
+    L = isp.lib()
+    F = FAKE_OUT
+
+    def call(w=64, h=64, pitch=64, mode=1, c=0, hc=0, mag=F, lap=F + (1 << 20), har=F + (2 << 20), dx=None,
+             op=64, inp=FAKE_IN):
+        return L.isp_pipeline_cfg3_u8(inp, w, h, pitch, mode, c, hc, 0, dx, None, mag, lap, har, op, 0, None)
+    assert call(w=0) == 1 and call(pitch=32) == 1 and call(op=32) == 1 and call(mode=4) == 1
+    assert call(mag=None) == 1 and call(lap=None) == 1 and call(har=None) == 1
+    assert call(c=256) == 1 and call(c=-1) == 1
+    assert call(hc=1021) == 1 and call(hc=-1021) == 1       # outside the Sobel range
+    assert call(mag=FAKE_IN + 100) == 3                     # EALIAS
+    assert call(dx=FAKE_IN + 64 * 63) == 3                  # int16 output overlapping the image tail

@@ -1,0 +1,106 @@
+"""GPU parity of the fused cfg3 pipeline (isp_pipeline_cfg3_u8) against
+the oracle COMPOSITION oracle.sobel -> oracle.laplace5_u8 -> oracle.harris: bit-exact on
+every output, every border mode, ISP (auto) and naive staging, ragged shapes spanning
+several 128x32 tiles, pitched images, and BASELINE.json configs[2] at full size.
+Harris' border handling applies to the dx/dy images (remapped coordinates), which the
+composition states by construction.
+"""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import synth
+
+pytestmark = pytest.mark.gpu
+
+MODES = ["clamp", "mirror", "repeat", "constant"]
+
+
+@pytest.fixture(scope="module")
+def isp():
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    import paper_conf_ipps_qiaoth21_b200 as m
+    m.lib()
+    oracle.build_oracle()
+    return m
+
+
+def dev(a):
+    return torch.from_numpy(np.ascontiguousarray(a)).cuda()
+
+
+def host(t):
+    torch.cuda.synchronize()
+    return t.cpu().numpy()
+
+
+def composition(img, mode, c, hc, thr):
+    rdx, rdy, rmag = oracle.sobel(img, mode, c)
+    return rdx, rdy, rmag, oracle.laplace5_u8(img, mode, c), oracle.harris(rdx, rdy, mode, hc, thr)
+
+
+@pytest.mark.parametrize("shape", [(1, 1), (2, 3), (5, 130), (33, 129), (64, 64), (70, 300), (131, 517)])
+@pytest.mark.parametrize("kind", ["structured", "noise"])
+def test_fused_matches_composition(isp, shape, kind):
+    h, w = shape
+    img = synth.structured_u8(h, w, 5) if kind == "structured" else synth.uniform_u8(h, w, 5)
+    d = dev(img)
+    for mode in MODES:
+        rdx, rdy, rmag, rlap, rhar = composition(img, mode, 45, -3, 0)
+        for v in ["auto", "naive"]:
+            dx = torch.empty((h, w), dtype=torch.int16, device="cuda")
+            dy = torch.empty_like(dx)
+            mag, lap, har = isp.isp_pipeline_cfg3_u8(d, mode, 45, -3, 0, dx=dx, dy=dy, variant=v)
+            for name, got, ref in [("dx", dx, rdx), ("dy", dy, rdy), ("mag", mag, rmag), ("lap", lap, rlap),
+                                   ("harris", har, rhar)]:
+                np.testing.assert_array_equal(host(got), ref, err_msg=f"{name} {mode} {v} {shape} {kind}")
+
+
+def test_fused_pitched_and_thresholds(isp):
+    h, w, pitch = 97, 333, 352
+    img = synth.uniform_u8(h, w, 9)
+    d = dev(synth.pitched(img, pitch, 200))
+    for mode in MODES:
+        for thr in [-(10 ** 12), 0, 10 ** 11]:
+            _, _, rmag, rlap, rhar = composition(img, mode, 7, 1020 if mode == "constant" else 0, thr)
+            mag = torch.zeros((h, pitch), dtype=torch.uint8, device="cuda")
+            lap, har = torch.zeros_like(mag), torch.zeros_like(mag)
+            isp.isp_pipeline_cfg3_u8(d, mode, 7, 1020 if mode == "constant" else 0, thr, mag=mag, lap=lap,
+                                     harris=har, w=w)
+            np.testing.assert_array_equal(host(mag)[:, :w], rmag, err_msg=f"mag {mode}")
+            np.testing.assert_array_equal(host(lap)[:, :w], rlap, err_msg=f"lap {mode}")
+            np.testing.assert_array_equal(host(har)[:, :w], rhar, err_msg=f"harris {mode} {thr}")
+            assert not host(mag)[:, w:].any()   # nothing written past the image width
+
+
+def test_fused_equals_three_launches(isp):
+    """Same bits as the unfused ISP pipeline on a multi-tile image (all modes)."""
+    img = synth.uniform_u8(300, 1000, 11)
+    d = dev(img)
+    for mode in MODES:
+        dx, dy, mag = isp.isp_sobel_u8(d, mode, 3)
+        lap = isp.isp_laplace5_u8(d, mode, 3)
+        har = isp.isp_harris_u8(dx, dy, mode, 5, 0)
+        fm, fl, fh = isp.isp_pipeline_cfg3_u8(d, mode, 3, 5, 0)
+        assert torch.equal(fm, mag) and torch.equal(fl, lap) and torch.equal(fh, har), mode
+
+
+def test_fused_cfg3_4096(isp):
+    """BASELINE.json configs[2] at full size, the launch bench_suite times: full-image
+    oracle for Sobel, sampled rows for Laplace and Harris."""
+    n = 4096
+    img = synth.structured_u8(n, n, synth.CONFIG_SEEDS["cfg3"])
+    rng = np.random.default_rng(3)
+    rows = sorted({0, 1, 2, 31, 32, n - 33, n - 32, n - 2, n - 1} | {int(r) for r in rng.integers(0, n, 24)})
+    d = dev(img)
+    dx = torch.empty((n, n), dtype=torch.int16, device="cuda")
+    dy = torch.empty_like(dx)
+    mag, lap, har = isp.isp_pipeline_cfg3_u8(d, "mirror", dx=dx, dy=dy)
+    rdx, rdy, rmag = oracle.sobel(img, "mirror", threads=8)
+    np.testing.assert_array_equal(host(dx), rdx)
+    np.testing.assert_array_equal(host(dy), rdy)
+    np.testing.assert_array_equal(host(mag), rmag)
+    np.testing.assert_array_equal(host(lap)[rows], oracle.laplace5_u8(img, "mirror", rows=rows))
+    np.testing.assert_array_equal(host(har)[rows], oracle.harris(rdx, rdy, "mirror", rows=rows))

@@ -144,8 +144,19 @@ def cfg3():
         tot = sum(x["us"] for x in r.values())
         r["pipeline"] = rec(tot, n * n, 13 * n * n)
         res[v] = r
+    # one-launch fusion (isp_pipeline_cfg3_u8): 1 B/px in, mag + lap + harris out
+    fused = {}
+    for v in ["auto", "naive"]:
+        us, _ = time_launch(lambda i: isp.isp_pipeline_cfg3_u8(imgs[i % nb], "mirror", mag=mags[i % nb],
+                                                               lap=laps[i % nb], harris=hars[i % nb], variant=v), nb)
+        fused[v] = rec(us, n * n, 4 * n * n)
+        us, _ = time_launch(lambda i: isp.isp_pipeline_cfg3_u8(imgs[i % nb], "mirror", mag=mags[i % nb],
+                                                               lap=laps[i % nb], harris=hars[i % nb], dx=dxs[i % nb],
+                                                               dy=dys[i % nb], variant=v), nb)
+        fused[v + "_with_dx_dy"] = rec(us, n * n, 8 * n * n)
+    fused["speedup_vs_3_launches"] = res["auto"]["pipeline"]["us"] / fused["auto"]["us"]
     return {"config": "Sobel + Laplace + Harris pipeline, 4096^2 u8, mirror (13 B/px: Sobel fused 6, Laplace 2, "
-                      "Harris 5)", "variants": res}
+                      "Harris 5; fused: 4 B/px, 8 with dx/dy)", "variants": res, "fused": fused}
 
 
 def cfg4(sweep=True):

@@ -23,7 +23,7 @@ def main():
     ap.add_argument("--size", type=int, default=4096)
     ap.add_argument("--window", type=int, default=5)
     ap.add_argument("--launches", type=int, default=4)
-    ap.add_argument("--op", default="gauss", choices=["gauss", "sobel", "laplace", "harris", "bilateral"])
+    ap.add_argument("--op", default="gauss", choices=["gauss", "sobel", "laplace", "harris", "bilateral", "fused3"])
     a = ap.parse_args()
     n = a.size
     if a.op != "gauss":
@@ -39,6 +39,9 @@ def main():
                 isp.isp_sobel_u8(u8, a.mode, dx=dx, dy=dy, mag=o8, variant=a.variant)
             elif a.op == "laplace":
                 isp.isp_laplace5_u8(u8, a.mode, out=o8, variant=a.variant)
+            elif a.op == "fused3":
+                lap, har = torch.empty_like(u8), torch.empty_like(u8)
+                isp.isp_pipeline_cfg3_u8(u8, a.mode, mag=o8, lap=lap, harris=har, variant=a.variant)
             elif a.op == "harris":
                 isp.isp_harris_u8(dx, dy, a.mode, out=o8, variant=a.variant)
             else:
