@@ -1,0 +1,113 @@
+#!/usr/bin/env python
+"""Paper-faithful sweeps on B200: ISP vs naive for the paper's five
+applications (Gaussian, Laplace, Sobel, Bilateral, Night) x four border modes x
+four image sizes (Fig. 6), with per-application geometric means (the Table IV analog),
+plus the image-size sweep 512..4096 step 256 of the Gaussian (Table III / Fig. 4 analog).
+
+Variants timed: naive (Eq. 3 baseline), warp (Listing 5), block (Listing 3), tma (Listing 3
+on the TMA-staged kernels, where built) and auto ("isp+m": the model decides, Eq. 10).
+Same methodology as tools/bench_suite.py (CUDA graph of 12 launches over rotating
+buffers, CUDA events on the launch stream).  Buffers rotate over >= 2x L2 only when 12
+pairs reach it: at 512^2 and 1024^2 the working set is L2-resident, like the paper's
+small images on its GPUs' caches.
+
+    python tools/paper_sweep.py > profiles/r01_paper_sweep.json
+"""
+from __future__ import annotations
+
+import json
+import math
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+sys.path.insert(0, os.path.dirname(os.path.abspath(__file__)))
+
+import numpy as np  # noqa: E402
+import torch  # noqa: E402
+
+import paper_conf_ipps_qiaoth21_b200 as isp  # noqa: E402
+import synth  # noqa: E402
+from bench_suite import nbuf_for, time_launch  # noqa: E402
+
+MODES = ["clamp", "mirror", "repeat", "constant"]
+VARIANTS = ["naive", "warp", "block", "tma", "auto"]
+SIZES = [512, 1024, 2048, 4096]
+G5 = np.outer(synth.binomial_row(5), synth.binomial_row(5)).astype(np.int32)
+
+
+def app_fns(n):
+    """(name, bytes per pixel moved, make_buffers(), launch(buf, mode, variant))."""
+    def u8_in():
+        return torch.from_numpy(synth.structured_u8(n, n, 3)).cuda()
+
+    def f32_in():
+        return torch.from_numpy(synth.structured_f32(n, n, 4)).cuda()
+
+    return [
+        ("gaussian_u8_5x5", 2, lambda: (u8_in(), torch.empty((n, n), dtype=torch.uint8, device="cuda")),
+         lambda b, m, v: isp.isp_filter_u8(b[0], G5, int(G5.sum()), m, 7, out=b[1], variant=v)),
+        ("laplace5_u8", 2, lambda: (u8_in(), torch.empty((n, n), dtype=torch.uint8, device="cuda")),
+         lambda b, m, v: isp.isp_laplace5_u8(b[0], m, 7, out=b[1], variant=v)),
+        ("sobel_u8", 6, lambda: (u8_in(), torch.empty((n, n), dtype=torch.int16, device="cuda"),
+                                 torch.empty((n, n), dtype=torch.int16, device="cuda"),
+                                 torch.empty((n, n), dtype=torch.uint8, device="cuda")),
+         lambda b, m, v: isp.isp_sobel_u8(b[0], m, 7, dx=b[1], dy=b[2], mag=b[3], variant=v)),
+        ("bilateral_f32_13x13", 8, lambda: (f32_in(), torch.empty((n, n), dtype=torch.float32, device="cuda")),
+         lambda b, m, v: isp.isp_bilateral_f32(b[0], 13, 3.0, 0.1, m, 0.5, out=b[1], variant=v)),
+        ("night_f32", 8, lambda: (f32_in(), torch.empty((n, n), dtype=torch.float32, device="cuda")),
+         lambda b, m, v: isp.isp_night_f32(b[0], m, 0.5, out=b[1], variant=v)),
+    ]
+
+
+def time_app(n, bpp, make, launch, mode, variant, bufs):
+    nb = len(bufs)
+    try:
+        us, plan = time_launch(lambda i: launch(bufs[i % nb], mode, variant), nb)
+    except isp.IspError as e:  # variant not built for this op (EUNSUPPORTED)
+        return {"unsupported": str(e)[:80]}
+    return {"us": round(us, 3), "mpix_s": round(n * n / us, 1), "choice": plan.get("choice") if plan else None,
+            "G": plan.get("g") if plan else None}
+
+
+def geo(xs):
+    xs = [x for x in xs if x and x > 0]
+    return math.exp(sum(math.log(x) for x in xs) / len(xs)) if xs else None
+
+
+def main():
+    out = {"device": torch.cuda.get_device_name(0), "apps": {}, "geomean": {}}
+    for n in SIZES:
+        for name, bpp, make, launch in app_fns(n):
+            nb = nbuf_for(bpp * n * n)
+            bufs = [make() for _ in range(nb)]
+            for mode in MODES:
+                r = {v: time_app(n, bpp, make, launch, mode, v, bufs) for v in VARIANTS}
+                base = r["naive"].get("us")
+                isp_us = [r[v]["us"] for v in ("warp", "block", "tma") if "us" in r[v]]
+                r["speedup_best_isp"] = base / min(isp_us) if base and isp_us else None
+                r["speedup_auto"] = base / r["auto"]["us"] if base and "us" in r["auto"] else None
+                out["apps"].setdefault(name, {}).setdefault(str(n), {})[mode] = r
+            del bufs
+            torch.cuda.empty_cache()
+        print(f"[sweep] {n} done", file=sys.stderr, flush=True)
+    for name, per in out["apps"].items():
+        best = [per[s][m]["speedup_best_isp"] for s in per for m in per[s]]
+        auto = [per[s][m]["speedup_auto"] for s in per for m in per[s]]
+        out["geomean"][name] = {"best_isp_vs_naive": geo(best), "auto_vs_naive": geo(auto),
+                                "min_auto_vs_naive": min(a for a in auto if a), "n": len(auto)}
+    # Table III / Fig. 4 analog: Gaussian size sweep, clamp, ISP (auto) vs naive
+    sweep = {}
+    for n in range(512, 4097, 256):
+        name, bpp, make, launch = app_fns(n)[0]
+        nb = nbuf_for(bpp * n * n)
+        bufs = [make() for _ in range(nb)]
+        sweep[str(n)] = {v: time_app(n, bpp, make, launch, "clamp", v, bufs) for v in ("naive", "auto")}
+        sweep[str(n)]["speedup_auto"] = sweep[str(n)]["naive"]["us"] / sweep[str(n)]["auto"]["us"]
+        del bufs
+    out["gaussian_size_sweep_clamp"] = sweep
+    print(json.dumps(out, indent=1))
+
+
+if __name__ == "__main__":
+    main()
