@@ -352,3 +352,21 @@ def test_strips_local_equal_full_image(isp, nranks, m):
                                                           variant=v))
                 got[y0:y0 + sh] = out
             np.testing.assert_array_equal(got, ref, err_msg=f"{mode} {v} P={nranks}")
+
+
+def test_auto_u8_calibrated_threshold(isp):
+    """Reading A29: launch-time AUTO takes the u8 streaming ISP kernel only when G > 2.4
+    (the measured B200 crossover), while isp_plan() keeps the paper's G > 1; results
+    stay identical to the oracle either way."""
+    g5 = np.outer(synth.binomial_row(5), synth.binomial_row(5)).astype(np.int32)
+    for n in (1024, 4096):
+        img = synth.structured_u8(n, n, 3)
+        out = isp.isp_filter_u8(dev(img), g5, int(g5.sum()), "clamp", 7)
+        torch.cuda.synchronize()
+        plan = isp.isp_last_plan()
+        if plan["g"] > 2.4:
+            assert plan["choice"] != 3, plan
+        elif not plan["degenerate"]:
+            assert plan["choice"] == 3, plan
+        rows = sample_rows(n, k=4, seed=n)
+        np.testing.assert_array_equal(host(out)[rows], oracle.filter_u8(img, g5, int(g5.sum()), "clamp", 7, rows=rows))
