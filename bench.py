@@ -127,21 +127,25 @@ class ClockSampler:
                 "reasons": reasons, "samples": len(rows)}
 
 
-def cpu_oracle_rate(target_s=12.0, threads=None):
-    """Oracle (oracle/ C, double accumulation, per-read border map) on the host cores over a
-    bounded row sample of the same workload, all four modes.  Returns dict for cpu_baseline."""
+def cpu_model():
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    import platform
+    return platform.processor() or "unknown"
+
+
+def _oracle_rows_rate(img, mask, threads, target_s):
+    """Oracle throughput (Mpixel/s) on a centred row band sized for ~target_s seconds."""
     import oracle
-    import synth
-    threads = threads or os.cpu_count() or 1
-    oracle.build_oracle()
-    img = synth.uniform_f32(N_SIDE, N_SIDE, synth.CONFIG_SEEDS["cfg2"])
-    mask = gauss_mask()
-    # calibrate on 4 rows per mode
     t = time.perf_counter()
     for m in MODES:
-        oracle.filter_f64(img, mask, m, CONST, rows=(0, 4 * threads), threads=threads)
+        oracle.filter_f64(img, mask, m, CONST, rows=(0, 2 * threads), threads=threads)
     dt = time.perf_counter() - t
-    rows = int(max(threads, min(N_SIDE, 4 * threads * target_s / max(dt, 1e-6))))
+    rows = int(max(threads, min(N_SIDE, 2 * threads * target_s / max(dt, 1e-6))))
     rows -= rows % threads
     rows = max(rows, threads)
     y0 = (N_SIDE - rows) // 2
@@ -150,9 +154,25 @@ def cpu_oracle_rate(target_s=12.0, threads=None):
         oracle.filter_f64(img, mask, m, CONST, rows=(y0, y0 + rows), threads=threads)
     dt = time.perf_counter() - t
     px = 4 * rows * N_SIDE
-    return {"value": px / dt / 1e6, "unit": UNIT, "cores": threads, "kind": "oracle",
-            "sample": f"rows [{y0},{y0 + rows}) of the 4096x4096 cfg2 image x 4 modes ({px} px, {dt:.1f} s)",
-            "seconds": dt}
+    return px / dt / 1e6, f"rows [{y0},{y0 + rows}) x 4 modes ({px} px, {dt:.1f} s)", dt
+
+
+def cpu_oracle_rate(target_s=8.0, threads=None):
+    """Oracle (oracle/ C, double accumulation, per-read border map) on the host cores over a
+    bounded row sample of the same workload, all four modes: once on 1 thread and once on
+    all cores.  `value` / `cores` are the all-core run."""
+    import oracle
+    import synth
+    threads = threads or os.cpu_count() or 1
+    oracle.build_oracle()
+    img = synth.uniform_f32(N_SIDE, N_SIDE, synth.CONFIG_SEEDS["cfg2"])
+    mask = gauss_mask()
+    v1, s1, d1 = _oracle_rows_rate(img, mask, 1, target_s / 2)
+    vn, sn, dn = _oracle_rows_rate(img, mask, threads, target_s)
+    return {"value": vn, "unit": UNIT, "cores": threads, "kind": "oracle",
+            "sample": f"cfg2 4096x4096 image, all cores: {sn}; 1 thread: {s1}",
+            "single_thread": {"value": v1, "unit": UNIT, "cores": 1, "sample": s1, "seconds": d1},
+            "cpu_model": cpu_model(), "seconds": dn + d1}
 
 
 # ------------------------------------------------------------------------------------------
@@ -185,7 +205,8 @@ def run_reference(args):
             "config": {"workload": "cfg2: 5x5 binomial Gaussian f32 4096x4096, 4 border modes (oracle sample)",
                        "sample_rows_per_step": rows_per_step},
             "cpu_baseline": {"value": val, "unit": UNIT, "cores": threads, "kind": "oracle",
-                             "sample": f"{rows_per_step} rows x 4096 px x 4 modes per step"},
+                             "sample": f"{rows_per_step} rows x 4096 px x 4 modes per step",
+                             "cpu_model": cpu_model()},
             "e2e": {"value": val, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 
@@ -249,35 +270,44 @@ def run_isp(args):
         for k in range(max(args.warmup, 1)):      # warm-up (also loads every kernel)
             step(k)
     torch.cuda.synchronize()
-    graphs = []          # graphs[ph]: one step of rotation phase ph (remainders)
-    graph_cycle = None   # one graph of a full rotation cycle (nphase steps, >= 12 launches)
+    # The timed region replays ONE graph holding exactly K steps (4K launches back to
+    # back, no inter-graph gaps); above MAX_GRAPH_STEPS steps it is a chunk graph of
+    # MAX_GRAPH_STEPS steps replayed, plus one graph for the remainder.
+    MAX_GRAPH_STEPS = 2000
+    chunk_graph, rem_graph, n_chunks = None, None, 0
+
+    def capture(nsteps, k0):
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g, stream=stream):
+            for k in range(k0, k0 + nsteps):
+                step(k)
+        return g
+
     if use_graph:
         try:
-            for ph in range(nphase):
-                g = torch.cuda.CUDAGraph()
-                with torch.cuda.graph(g, stream=stream):
-                    step(ph)
-                graphs.append(g)
-            graph_cycle = torch.cuda.CUDAGraph()
-            with torch.cuda.graph(graph_cycle, stream=stream):
-                for ph in range(nphase):
-                    step(ph)
-            for g in graphs + [graph_cycle]:
-                g.replay()
+            chunk = min(args.steps, MAX_GRAPH_STEPS)
+            chunk -= chunk % nphase if args.steps > MAX_GRAPH_STEPS else 0
+            n_chunks = args.steps // chunk
+            chunk_graph = capture(chunk, 0)
+            rem = args.steps - n_chunks * chunk
+            rem_graph = capture(rem, n_chunks * chunk) if rem else None
+            for g in (chunk_graph, rem_graph):
+                if g is not None:
+                    g.replay()
             torch.cuda.synchronize()
         except Exception as e:  # pragma: no cover
             print(f"[bench] graph capture failed ({e}); eager launches", file=sys.stderr)
-            graphs, graph_cycle = [], None
+            chunk_graph, rem_graph = None, None
             use_graph = False
 
     def run_steps(K, v=variant):
-        """Exactly K steps: K // nphase replays of the cycle graph + the remaining steps."""
+        """Exactly K steps (K == args.steps when graphs are used)."""
         with torch.cuda.stream(stream):
-            if use_graph and v == variant:
-                for _ in range(K // nphase):
-                    graph_cycle.replay()
-                for k in range(K % nphase):
-                    graphs[k].replay()
+            if use_graph and v == variant and K == args.steps:
+                for _ in range(n_chunks):
+                    chunk_graph.replay()
+                if rem_graph is not None:
+                    rem_graph.replay()
             else:
                 for k in range(K):
                     step(k, v)
@@ -318,7 +348,7 @@ def run_isp(args):
             "kernel": f"variant {args.variant}: " + ("k_staged<OpSepF32<5,5>> (TMA-staged ISP)" if plan["choice"] == 4 else "k_stencil<OpSepF32<5,5>>"),
             "algorithmic_bytes_per_launch": BYTES_PER_PX * N_SIDE * N_SIDE,
             "duration_us": per_launch_us,
-            "duration_method": "timed region / launches (CUDA-graph replay of a full rotation cycle, kernels back-to-back)"}
+            "duration_method": "timed region / launches (one CUDA graph of the K steps, kernels back to back)"}
 
     # ---- ISP vs naive per mode (same methodology, single-GPU variants) ----
     variants = {}

@@ -109,7 +109,12 @@ isp_status_t isp_laplace5_u8(const uint8_t *img, int w, int h, int pitch, int bo
 /* Harris response over Sobel derivatives (BASELINE.json configs[2]; not in the paper;
  * a10): 3x3 window, weights [1,2,1](x)[1,2,1]; Sxx, Syy, Sxy exact;
  * R25 = 25*(Sxx*Syy - Sxy^2) - (Sxx+Syy)^2 (k = 1/25, int64); out = R25 > thr ? 255 : 0.
- * dx, dy share `pitch`; border handling applies to the dx/dy images (const_val int16). */
+ * dx, dy share `pitch`; border handling applies to the dx/dy images.
+ * Domain (precondition): every dx, dy value and const_val lie in [-1020, 1020], the
+ * range of 3x3 Sobel derivatives of u8 images.  Inside it the kernels evaluate R25
+ * exactly (f32 window sums < 2^24, f64 response < 2^53)
+ * and equal the int64 definition bit for bit at every thr.  const_val outside the
+ * range returns ISP_EINVAL; device data outside it is not checked (results unspecified). */
 isp_status_t isp_harris_u8(const int16_t *dx, const int16_t *dy, int w, int h, int pitch, int border_mode,
                            int const_val, int64_t thr, uint8_t *out, int out_pitch, isp_variant_t variant,
                            isp_stream_t stream);
@@ -231,6 +236,11 @@ isp_status_t isp_shard_filter_u8(isp_shard_ctx *ctx, uint8_t *strip, int w, int 
 isp_status_t isp_shard_filter_local_f32(float *strip, int w, int H, int pitch, int halo, int rank, int nranks,
                                         const float *mask, int mw, int mh, int border_mode, float const_val,
                                         float *out, int out_pitch, isp_variant_t variant, isp_stream_t stream);
+/* u8 counterpart of isp_shard_filter_local_f32 (the launch part of isp_shard_filter_u8). */
+isp_status_t isp_shard_filter_local_u8(uint8_t *strip, int w, int H, int pitch, int halo, int rank, int nranks,
+                                       const int32_t *mask, int mw, int mh, int32_t divisor, int border_mode,
+                                       int const_val, uint8_t *out, int out_pitch, isp_variant_t variant,
+                                       isp_stream_t stream);
 isp_status_t isp_shard_destroy(isp_shard_ctx *ctx);
 
 /* Tuning: force the launch shape (warps per block along x, tile height in rows);
@@ -239,6 +249,11 @@ isp_status_t isp_set_launch_override(int warps_x, int tile_h);
 
 /* Last launch's resolved plan on this thread (which variant/tile AUTO picked). */
 isp_status_t isp_last_plan(isp_plan_info *out);
+/* The last min(n, 16) resolved launch plans of this thread, oldest first (multi-launch
+ * calls: isp_night_f32, isp_shard_*); returns how many were written.
+ * isp_clear_plans forgets them (tests). */
+int isp_recent_plans(isp_plan_info *out, int n);
+void isp_clear_plans(void);
 const char *isp_status_string(isp_status_t s);
 const char *isp_last_error(void); /* thread-local */
 int isp_version(void);

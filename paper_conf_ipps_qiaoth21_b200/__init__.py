@@ -24,9 +24,11 @@ __all__ = [
     "lib", "IspError", "PlanInfo", "ModelParams",
     "isp_filter", "isp_filter_naive", "isp_filter_ex", "isp_filter_sep_f32", "isp_filter_u8",
     "isp_sobel_u8", "isp_laplace5_u8", "isp_harris_u8", "isp_pipeline_cfg3_u8", "isp_bilateral_f32", "isp_atrous_f32",
-    "isp_night_f32", "isp_plan", "isp_model_defaults", "isp_last_plan", "isp_set_launch_override",
+    "isp_night_f32", "isp_plan", "isp_model_defaults", "isp_last_plan", "isp_recent_plans", "isp_clear_plans",
+    "isp_set_launch_override",
     "isp_shard_unique_id", "isp_shard_init", "isp_shard_rows", "isp_shard_schedule",
-    "isp_shard_filter_f32", "isp_shard_filter_u8", "isp_shard_filter_local_f32", "isp_shard_destroy",
+    "isp_shard_filter_f32", "isp_shard_filter_u8", "isp_shard_filter_local_f32", "isp_shard_filter_local_u8",
+    "isp_shard_destroy",
 ]
 
 CLAMP, MIRROR, REPEAT, CONSTANT = 0, 1, 2, 3
@@ -111,6 +113,8 @@ _SIGS = {
     "isp_shard_filter_u8": [_P, _P, _I, _I, _I, _I, _P, _I, _I, ctypes.c_int32, _I, _I, _P, _I, _I, _P, _P],
     "isp_shard_destroy": [_P],
     "isp_shard_filter_local_f32": [_P, _I, _I, _I, _I, _I, _I, _P, _I, _I, _I, _F, _P, _I, _I, _P],
+    "isp_shard_filter_local_u8": [_P, _I, _I, _I, _I, _I, _I, _P, _I, _I, ctypes.c_int32, _I, _I, _P, _I, _I, _P],
+    "isp_recent_plans": [_P, _I],
 }
 
 _lib = None
@@ -133,6 +137,8 @@ def lib():
         L.isp_status_string.restype = ctypes.c_char_p
         L.isp_status_string.argtypes = [ctypes.c_int]
         L.isp_version.restype = ctypes.c_int
+        L.isp_clear_plans.restype = None
+        L.isp_clear_plans.argtypes = []
         _lib = L
     return _lib
 
@@ -163,13 +169,30 @@ def _img(t, dtype, name="img"):
 
 def _geom(img, w):
     h, pitch = img.shape
-    return (pitch if w is None else int(w)), h, pitch
+    w = pitch if w is None else int(w)
+    if w > pitch:
+        raise ValueError(f"width {w} exceeds the buffer's row pitch {pitch}")
+    return w, h, pitch
 
 
-def _out(out, img, w, dtype):
+def _out(out, img, w, dtype, rows=None, name="out"):
+    """Caller-supplied output: right dtype, contiguous 2-D, on img's device, at least
+    `rows` (default: img's) rows and w columns -- checked here because the C ABI takes
+    raw pointers and cannot see the allocation."""
+    rows = img.shape[0] if rows is None else rows
     if out is None:
-        return torch.empty((img.shape[0], w), dtype=dtype, device=img.device)
-    return _img(out, dtype, "out")
+        return torch.empty((rows, w), dtype=dtype, device=img.device)
+    _img(out, dtype, name)
+    if out.device != img.device:
+        raise ValueError(f"{name} is on {out.device}, input on {img.device}")
+    if out.shape[0] < rows or out.shape[1] < w:
+        raise ValueError(f"{name} has shape {tuple(out.shape)}, needs at least ({rows}, {w})")
+    return out
+
+
+def _in_geom(t, w, h, name):
+    if t.shape[0] < h or t.shape[1] < w:
+        raise ValueError(f"{name} has shape {tuple(t.shape)}, needs at least ({h}, {w})")
 
 
 def _stream(t, stream=None):
@@ -239,9 +262,11 @@ def isp_sobel_u8(img, border_mode, const_val=0, dx=None, dy=None, mag=None, vari
     if mag is None and "mag" in want:
         mag = torch.empty((h, w), dtype=torch.uint8, device=img.device)
     op = next(t for t in (dx, dy, mag) if t is not None).shape[1]
-    for t in (dx, dy, mag):
-        if t is not None and t.shape[1] != op:
-            raise ValueError("dx, dy and mag must share out_pitch")
+    for t, dt, nm in ((dx, torch.int16, "dx"), (dy, torch.int16, "dy"), (mag, torch.uint8, "mag")):
+        if t is not None:
+            _out(t, img, w, dt, name=nm)
+            if t.shape[1] != op:
+                raise ValueError("dx, dy and mag must share out_pitch")
     ptr = lambda t: t.data_ptr() if t is not None else None  # noqa: E731
     _check(lib().isp_sobel_u8(img.data_ptr(), w, h, pitch, _mode(border_mode), int(const_val), ptr(dx), ptr(dy),
                               ptr(mag), op, _variant(variant), _stream(img, stream)))
@@ -281,7 +306,7 @@ def isp_pipeline_cfg3_u8(img, border_mode, const_val=0, harris_const=0, thr=0, m
     op = mag.shape[1]
     for t, dt in ((lap, torch.uint8), (harris, torch.uint8), (dx, torch.int16), (dy, torch.int16)):
         if t is not None:
-            _img(t, dt, "out")
+            _out(t, img, w, dt)
             if t.shape[1] != op:
                 raise ValueError("all outputs must share out_pitch")
     ptr = lambda t: t.data_ptr() if t is not None else None  # noqa: E731
@@ -346,6 +371,17 @@ def isp_last_plan():
     return info.as_dict()
 
 
+def isp_recent_plans(n=16):
+    """The last min(n, 16) launch plans of this thread, oldest first."""
+    arr = (PlanInfo * 16)()
+    k = lib().isp_recent_plans(arr, min(int(n), 16))
+    return [arr[i].as_dict() for i in range(k)]
+
+
+def isp_clear_plans():
+    lib().isp_clear_plans()
+
+
 def isp_set_launch_override(warps_x=0, tile_h=0):
     _check(lib().isp_set_launch_override(int(warps_x), int(tile_h)))
 
@@ -361,6 +397,7 @@ def isp_shard_init(uid: bytes, rank, nranks, device):
     ctx = ctypes.c_void_p()
     buf = (ctypes.c_ubyte * 128).from_buffer_copy(uid)
     _check(lib().isp_shard_init(ctypes.byref(ctx), buf, int(rank), int(nranks), int(device)))
+    _CTX_RANKS[ctx.value] = (int(rank), int(nranks))
     return ctx
 
 
@@ -377,14 +414,36 @@ def isp_shard_schedule(H, rank, nranks, halo, hy, border_mode):
     return sc.as_dict()
 
 
+def _strip_rows(strip, H, halo, rank, nranks, hy):
+    """Check the strip buffer holds strip_h + 2*halo rows (include/isp.h) before the C ABI
+    writes halo rows into it; returns strip_h."""
+    if halo < hy:
+        raise ValueError(f"halo {halo} < window half-height {hy}")
+    _, sh = isp_shard_rows(H, rank, nranks)
+    if strip.shape[0] != sh + 2 * halo:
+        raise ValueError(f"strip has {strip.shape[0]} rows, rank {rank}/{nranks} of H={H} needs "
+                         f"strip_h + 2*halo = {sh + 2 * halo}")
+    return sh
+
+
+_CTX_RANKS = {}
+
+
+def _ctx_ranks(ctx, rank, nranks):
+    if rank is None or nranks is None:
+        rank, nranks = _CTX_RANKS[ctx.value]
+    return int(rank), int(nranks)
+
+
 def isp_shard_filter_f32(ctx, strip, H, halo, mask, border_mode, const_val=0.0, out=None, variant=AUTO, w=None,
-                         stream=None, comm_stream=None):
+                         stream=None, comm_stream=None, rank=None, nranks=None):
     _img(strip, torch.float32, "strip")
     w, _, pitch = _geom(strip, w)
     m, mp = _host(mask, ctypes.c_float)
     mh, mw = m.shape
-    if out is None:
-        out = torch.empty((strip.shape[0] - 2 * halo, w), dtype=torch.float32, device=strip.device)
+    rank, nranks = _ctx_ranks(ctx, rank, nranks)
+    sh = _strip_rows(strip, H, halo, rank, nranks, mh // 2)
+    out = _out(out, strip, w, torch.float32, rows=sh)
     cs = comm_stream if comm_stream is not None else torch.cuda.current_stream(strip.device)
     _check(lib().isp_shard_filter_f32(ctx, strip.data_ptr(), w, int(H), pitch, int(halo), mp, mw, mh,
                                       _mode(border_mode), float(const_val), out.data_ptr(), out.shape[1],
@@ -393,13 +452,14 @@ def isp_shard_filter_f32(ctx, strip, H, halo, mask, border_mode, const_val=0.0, 
 
 
 def isp_shard_filter_u8(ctx, strip, H, halo, mask, divisor, border_mode, const_val=0, out=None, variant=AUTO, w=None,
-                        stream=None, comm_stream=None):
+                        stream=None, comm_stream=None, rank=None, nranks=None):
     _img(strip, torch.uint8, "strip")
     w, _, pitch = _geom(strip, w)
     m, mp = _host(mask, ctypes.c_int32)
     mh, mw = m.shape
-    if out is None:
-        out = torch.empty((strip.shape[0] - 2 * halo, w), dtype=torch.uint8, device=strip.device)
+    rank, nranks = _ctx_ranks(ctx, rank, nranks)
+    sh = _strip_rows(strip, H, halo, rank, nranks, mh // 2)
+    out = _out(out, strip, w, torch.uint8, rows=sh)
     cs = comm_stream if comm_stream is not None else torch.cuda.current_stream(strip.device)
     _check(lib().isp_shard_filter_u8(ctx, strip.data_ptr(), w, int(H), pitch, int(halo), mp, mw, mh, int(divisor),
                                      _mode(border_mode), int(const_val), out.data_ptr(), out.shape[1],
@@ -414,11 +474,26 @@ def isp_shard_filter_local_f32(strip, H, halo, rank, nranks, mask, border_mode, 
     w, _, pitch = _geom(strip, w)
     m, mp = _host(mask, ctypes.c_float)
     mh, mw = m.shape
-    if out is None:
-        out = torch.empty((strip.shape[0] - 2 * halo, w), dtype=torch.float32, device=strip.device)
+    sh = _strip_rows(strip, H, halo, rank, nranks, mh // 2)
+    out = _out(out, strip, w, torch.float32, rows=sh)
     _check(lib().isp_shard_filter_local_f32(strip.data_ptr(), w, int(H), pitch, int(halo), int(rank), int(nranks), mp,
                                             mw, mh, _mode(border_mode), float(const_val), out.data_ptr(),
                                             out.shape[1], _variant(variant), _stream(strip, stream)))
+    return out
+
+
+def isp_shard_filter_local_u8(strip, H, halo, rank, nranks, mask, divisor, border_mode, const_val=0, out=None,
+                              variant=AUTO, w=None, stream=None):
+    """u8 strip launches of one rank without communication (halo rows already filled)."""
+    _img(strip, torch.uint8, "strip")
+    w, _, pitch = _geom(strip, w)
+    m, mp = _host(mask, ctypes.c_int32)
+    mh, mw = m.shape
+    sh = _strip_rows(strip, H, halo, rank, nranks, mh // 2)
+    out = _out(out, strip, w, torch.uint8, rows=sh)
+    _check(lib().isp_shard_filter_local_u8(strip.data_ptr(), w, int(H), pitch, int(halo), int(rank), int(nranks), mp,
+                                           mw, mh, int(divisor), _mode(border_mode), int(const_val), out.data_ptr(),
+                                           out.shape[1], _variant(variant), _stream(strip, stream)))
     return out
 
 

@@ -22,6 +22,10 @@ namespace {
 
 thread_local char g_err[512] = "";
 thread_local isp_plan_info g_last_plan{};
+// the last kRecent resolved plans of this thread (multi-launch calls: Night, strips)
+constexpr int kRecent = 16;
+thread_local isp_plan_info g_recent[kRecent];
+thread_local long long g_n_plans = 0;
 int g_override_wx = 0, g_override_ty = 0;
 
 // Rows of the strips holding the image's top / bottom border in a balanced split, in
@@ -443,6 +447,7 @@ isp_status_t resolve_and_launch(Desc &d, int fam, int w, int h, int mw, int mh, 
     if (getenv("ISP_CTA_TRACE")) d.g.trace = cta_trace_buffer();
     d.g.edge_w = p.edge_w;
     g_last_plan = info;
+    g_recent[g_n_plans++ % kRecent] = info;
     cudaError_t e = run(d);
     if (e == cudaSuccess) e = cudaGetLastError();
     return cuda_status(e, what);
@@ -569,6 +574,21 @@ isp_status_t isp_last_plan(isp_plan_info *out)
     if (!out) return fail(ISP_EINVAL, "null output");
     *out = g_last_plan;
     return ISP_OK;
+}
+
+int isp_recent_plans(isp_plan_info *out, int n)
+{
+    if (!out || n <= 0) return 0;
+    const int avail = (int)std::min<long long>(g_n_plans, kRecent);
+    const int k = std::min(n, avail);
+    for (int i = 0; i < k; ++i) out[i] = g_recent[(g_n_plans - k + i) % kRecent];  // oldest first
+    return k;
+}
+
+void isp_clear_plans(void)
+{
+    g_n_plans = 0;
+    g_last_plan = isp_plan_info{};
 }
 
 // Launch-shape override for tuning sweeps (0 = planner default).  Not thread-safe.
@@ -777,7 +797,10 @@ isp_status_t isp_harris_u8(const int16_t *dx, const int16_t *dy, int w, int h, i
     isp_status_t s = check_geom(w, h, pitch, out_pitch, 3, 3, border_mode);
     if (s != ISP_OK) return s;
     if (!dx || !dy || !out) return fail(ISP_EINVAL, "null pointer");
-    if (const_val < -32768 || const_val > 32767) return fail(ISP_EINVAL, "int16 constant %d", const_val);
+    // exact only inside the range of 3x3 Sobel derivatives of u8 images (isp.h): the
+    // f32 window sums / f64 response of OpHarris are exact for |v| <= 1020
+    if (const_val < -1020 || const_val > 1020)
+        return fail(ISP_EINVAL, "harris constant %d outside the Sobel range [-1020,1020]", const_val);
     const size_t ob = img_bytes(w, h, out_pitch, 1);
     if (ranges_overlap(dx, img_bytes(w, h, pitch, 2), out, ob) || ranges_overlap(dy, img_bytes(w, h, pitch, 2), out, ob))
         return fail(ISP_EALIAS, "input and output overlap");

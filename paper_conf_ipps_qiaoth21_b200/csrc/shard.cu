@@ -197,6 +197,20 @@ isp_status_t isp_shard_filter_local_f32(float *strip, int w, int H, int pitch, i
                             (cudaStream_t)stream, (cudaStream_t)stream, f);
 }
 
+isp_status_t isp_shard_filter_local_u8(uint8_t *strip, int w, int H, int pitch, int halo, int rank, int nranks,
+                                       const int32_t *mask, int mw, int mh, int32_t divisor, int border_mode,
+                                       int const_val, uint8_t *out, int out_pitch, isp_variant_t variant,
+                                       isp_stream_t stream)
+{
+    if (!strip || !out || !mask) return ispi_fail(ISP_EINVAL, "null pointer");
+    auto f = [&](const uint8_t *in_base, uint8_t *o, const RowRange &rr) {
+        return ispi_filter_u8(in_base, w, H, pitch, mask, mw, mh, divisor, border_mode, const_val, o, out_pitch,
+                              variant, stream, &rr);
+    };
+    return shard_run<uint8_t>(nullptr, rank, nranks, strip, w, H, pitch, halo, mh / 2, border_mode, out, out_pitch,
+                              (cudaStream_t)stream, (cudaStream_t)stream, f);
+}
+
 isp_status_t isp_shard_destroy(isp_shard_ctx *ctx)
 {
     if (!ctx) return ISP_OK;

@@ -1,0 +1,423 @@
+"""GPU parity of every ISP region body against the oracle, with proof that the body ran.
+
+The round-1 parity shapes mostly sent compiled-window launches to the NAIVE kernel
+(misaligned widths, degenerate tiles), so ISP bodies were compared only with naive.
+Here every shape is vector/TMA aligned (f32: width % 4 == 0; u8: width % 16 == 0),
+spans several tile columns plus a partial last tile and several tile rows, and each
+launch is checked through isp_last_plan() / isp_recent_plans():
+
+  * the requested variant is the one that ran (TMA -> k_staged / k_tile, WARP ->
+    Listing 5, BLOCK -> Listing 3, NAIVE), and
+  * the plan is not degenerate (reading A3), so the nine-region dispatch ran.
+
+Then the output must equal the oracle: bit-exact for integer / byte outputs, A28 for
+f32 (|g - o| <= 1e-5 * max(|o|, sum |w * in|)), max-abs 1e-4 for the Bilateral, and
+every variant bitwise equal to NAIVE (ISP == NAIVE invariant).
+"""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import synth
+
+pytestmark = pytest.mark.gpu
+
+MODES = ["clamp", "mirror", "repeat", "constant"]
+CODE = {"auto": 0, "block": 1, "warp": 2, "naive": 3, "tma": 4}
+ISP_VARIANTS = ["tma", "warp", "block"]
+
+# (h, w): aligned, >= 3 tile columns + a partial one, several tile rows
+F32_SHAPES = [(70, 2052), (45, 4100)]
+U8_SHAPES = [(70, 2064), (33, 4112)]
+
+
+@pytest.fixture(scope="module")
+def isp():
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    import paper_conf_ipps_qiaoth21_b200 as m
+    m.lib()
+    oracle.build_oracle()
+    return m
+
+
+def dev(a):
+    return torch.from_numpy(np.ascontiguousarray(a)).cuda()
+
+
+def host(t):
+    torch.cuda.synchronize()
+    return t.cpu().numpy()
+
+
+def check_f32(got, ref, scale, tol=1e-5):
+    bound = tol * np.maximum(np.abs(ref), scale) + 1e-30
+    err = np.abs(got.astype(np.float64) - ref)
+    bad = err > bound
+    assert not bad.any(), f"{bad.sum()} px off; worst err {err.max():.3e} at {np.unravel_index(err.argmax(), err.shape)}"
+
+
+def ran(isp, v, has_tma=True):
+    """Assert the last launch ran variant v on a non-degenerate plan; return the plan."""
+    p = isp.isp_last_plan()
+    assert not p["degenerate"], f"degenerate plan for {v}: {p}"
+    want = CODE[v]
+    if v == "tma" and not has_tma:
+        want = CODE["block"]
+    if v != "auto":
+        assert p["choice"] == want, f"requested {v}, ran choice {p['choice']} ({p})"
+    return p
+
+
+def run_all(isp, call, has_tma=True):
+    """Run call(v) for naive + the ISP variants + auto; return {v: host array}."""
+    outs = {}
+    for v in ["naive"] + ISP_VARIANTS + ["auto"]:
+        r = call(v)
+        ran(isp, v, has_tma)
+        outs[v] = host(r) if not isinstance(r, tuple) else tuple(host(t) for t in r)
+    return outs
+
+
+def binomial_f32(m):
+    b = synth.binomial_row(m).astype(np.float64)
+    return (np.outer(b, b) / b.sum() ** 2).astype(np.float32)
+
+
+# ---------------------------------------------------------------- f32, compiled windows
+@pytest.mark.parametrize("mask_kind", ["binomial3", "binomial5", "binomial7", "rand3", "rand5", "rand7"])
+@pytest.mark.parametrize("shape", F32_SHAPES)
+def test_f32_compiled_bodies(isp, shape, mask_kind):
+    """OpSepF32<3/5/7> (rank-1 masks) and OpConvF32<3/5/7> in k_staged, k_stencil
+    Listing 3 / Listing 5 bodies and naive, every border mode."""
+    h, w = shape
+    img = synth.uniform_f32(h, w, 100 + h)
+    m = int(mask_kind[-1])
+    mask = binomial_f32(m) if mask_kind.startswith("binomial") else \
+        np.random.default_rng(m).standard_normal((m, m)).astype(np.float32)
+    d = dev(img)
+    for mode in MODES:
+        ref, sc = oracle.filter_f64(img, mask, mode, 0.375, with_scale=True)
+        outs = run_all(isp, lambda v: isp.isp_filter_ex(d, mask, mode, 0.375, variant=v))
+        for v, o in outs.items():
+            check_f32(o, ref, sc)
+            np.testing.assert_array_equal(o, outs["naive"], err_msg=f"{v} != naive ({mode} {mask_kind})")
+
+
+@pytest.mark.parametrize("m", [3, 5, 7])
+def test_f32_separable_entry_bodies(isp, m):
+    h, w = F32_SHAPES[0]
+    img = synth.uniform_f32(h, w, 5)
+    rng = np.random.default_rng(m)
+    row, col = rng.standard_normal(m).astype(np.float32), rng.standard_normal(m).astype(np.float32)
+    mask = np.outer(col.astype(np.float64), row.astype(np.float64))
+    d = dev(img)
+    for mode in MODES:
+        ref, sc = oracle.filter_f64(img, mask, mode, -1.5, with_scale=True)
+        outs = run_all(isp, lambda v: isp.isp_filter_sep_f32(d, row, col, mode, -1.5, variant=v))
+        for v, o in outs.items():
+            check_f32(o, ref, sc)
+            np.testing.assert_array_equal(o, outs["naive"])
+
+
+# ---------------------------------------------------------------- f32, runtime windows (direct / tiled)
+@pytest.mark.parametrize("mask_kind", ["rand9", "rand5x3", "rand1x7", "rand13", "rand31"])
+def test_f32_direct_bodies(isp, mask_kind):
+    h, w = 70, 1036
+    img = synth.uniform_f32(h, w, 41)
+    dims = mask_kind[4:]
+    mh, mw = (int(dims), int(dims)) if "x" not in dims else map(int, dims.split("x"))
+    mask = np.random.default_rng(mh * 31 + mw).standard_normal((mh, mw)).astype(np.float32)
+    d = dev(img)
+    for mode in MODES:
+        ref, sc = oracle.filter_f64(img, mask, mode, 0.25, with_scale=True)
+        outs = run_all(isp, lambda v: isp.isp_filter_ex(d, mask, mode, 0.25, variant=v))
+        for v, o in outs.items():
+            check_f32(o, ref, sc)
+            np.testing.assert_array_equal(o, outs["naive"], err_msg=f"{v} {mode} {mask_kind}")
+
+
+# ---------------------------------------------------------------- u8 operators
+@pytest.mark.parametrize("mask_kind", ["gauss3", "gauss5", "gauss7", "rand3", "rand5", "rand7", "laplace5", "rand9"])
+@pytest.mark.parametrize("shape", U8_SHAPES)
+def test_u8_bodies(isp, shape, mask_kind):
+    """OpSepU8 / OpConvU8 in k_staged (u8 TMA), k_stencil Listing 3 / 5 and naive; the
+    direct family for 9x9."""
+    h, w = shape
+    img = synth.uniform_u8(h, w, 200 + w)
+    if mask_kind.startswith("gauss"):
+        mask, div = oracle.gaussian_u8_mask(int(mask_kind[-1]))
+    elif mask_kind == "laplace5":
+        mask, div = oracle.LAPLACE5, 1
+    else:
+        k = int(mask_kind[-1])
+        mask, div = np.random.default_rng(k).integers(-9, 10, (k, k)).astype(np.int32), 7 + k
+    d = dev(img)
+    for mode in MODES:
+        ref = oracle.filter_u8(img, mask, div, mode, 77)
+        outs = run_all(isp, lambda v: isp.isp_filter_u8(d, mask, div, mode, 77, variant=v),
+                       has_tma=mask_kind != "rand9")   # no tiled kernel for runtime-window u8
+        for v, o in outs.items():
+            np.testing.assert_array_equal(o, ref, err_msg=f"{mask_kind} {mode} {v}")
+
+
+@pytest.mark.parametrize("shape", U8_SHAPES)
+def test_sobel_laplace_harris_bodies(isp, shape):
+    """OpSobel, OpLaplace5 and OpHarris bodies (T/B/L/R/corners/Body) in every mode,
+    streaming and TMA-staged."""
+    h, w = shape
+    img = synth.structured_u8(h, w, 11)
+    d = dev(img)
+    for mode in MODES:
+        rdx, rdy, rmag = oracle.sobel(img, mode, 45)
+        rlap = oracle.laplace5_u8(img, mode, 45)
+        rhar = oracle.harris(rdx, rdy, mode, -3, 0)
+        sob = run_all(isp, lambda v: isp.isp_sobel_u8(d, mode, 45, variant=v))
+        for v, (dx, dy, mag) in sob.items():
+            np.testing.assert_array_equal(dx, rdx, err_msg=f"dx {mode} {v}")
+            np.testing.assert_array_equal(dy, rdy, err_msg=f"dy {mode} {v}")
+            np.testing.assert_array_equal(mag, rmag, err_msg=f"mag {mode} {v}")
+        lap = run_all(isp, lambda v: isp.isp_laplace5_u8(d, mode, 45, variant=v))
+        for v, o in lap.items():
+            np.testing.assert_array_equal(o, rlap, err_msg=f"laplace {mode} {v}")
+        ddx, ddy = dev(rdx), dev(rdy)
+        har = run_all(isp, lambda v: isp.isp_harris_u8(ddx, ddy, mode, -3, 0, variant=v))
+        for v, o in har.items():
+            np.testing.assert_array_equal(o, rhar, err_msg=f"harris {mode} {v}")
+
+
+# ---------------------------------------------------------------- Bilateral
+@pytest.mark.parametrize("win", [3, 13, 31])
+def test_bilateral_bodies(isp, win):
+    h, w = 70, 1036
+    img = synth.structured_f32(h, w, 4)
+    sd = (win - 1) / 4.0
+    d = dev(img)
+    for mode in MODES:
+        ref = oracle.bilateral(img, win, sd, 0.1, mode, 0.5)
+        outs = run_all(isp, lambda v: isp.isp_bilateral_f32(d, win, sd, 0.1, mode, 0.5, variant=v))
+        for v, o in outs.items():
+            assert np.abs(o - ref).max() <= 1e-4, (mode, v)
+            np.testing.assert_array_equal(o, outs["naive"], err_msg=f"{v} {mode}")
+
+
+# ---------------------------------------------------------------- Atrous / Night
+@pytest.mark.parametrize("dil", [1, 2, 4, 8])
+@pytest.mark.parametrize("shape", F32_SHAPES)
+def test_atrous_bodies(isp, shape, dil):
+    """Row-direct Atrous bodies incl. Body/T/B; no TMA kernel (TMA request runs BLOCK).
+    Tolerance A28: the weights are non-negative and the data (and C) non-negative, so
+    sum |w * in| = |o| and the bound is 1e-5 |o|."""
+    h, w = shape
+    img = synth.uniform_f32(h, w, 17)
+    t = dev(img)
+    for mode in MODES:
+        ref = oracle.atrous(img, dil, mode, 0.75)
+        outs = run_all(isp, lambda v: isp.isp_atrous_f32(t, dil, mode, 0.75, variant=v), has_tma=False)
+        for v, o in outs.items():
+            check_f32(o, ref, np.abs(ref))
+            np.testing.assert_array_equal(o, outs["naive"])
+
+
+def test_night_bodies(isp):
+    """Night = Atrous d=1,2,4,8 + tone map, each pass non-degenerate ISP (isp_recent_plans).
+    Each pass is within A28 of its exactly-rounded value and the passes are averages with
+    non-negative weights (errors do not grow), so 4 passes stay within 4e-5 |o|."""
+    h, w = F32_SHAPES[0]
+    img = synth.uniform_f32(h, w, 4)
+    d = dev(img)
+    for mode in MODES:
+        ref = oracle.night(img, mode, 0.25)
+        outs = {}
+        for v in ["naive", "warp", "block", "auto"]:
+            isp.isp_clear_plans()
+            outs[v] = host(isp.isp_night_f32(d, mode, 0.25, variant=v))
+            plans = isp.isp_recent_plans()
+            assert len(plans) == 4
+            for p in plans:
+                assert not p["degenerate"]
+                if v != "auto":
+                    assert p["choice"] == CODE[v]
+        for v, o in outs.items():
+            check_f32(o, ref, np.abs(ref), tol=4e-5)
+            np.testing.assert_array_equal(o, outs["naive"])
+
+
+# ---------------------------------------------------------------- multi-GPU strips (RowRange ISP)
+def _strip_run(isp, img, H, W, halo, hy, nranks, r, mode, fill, local_call):
+    sc = isp.isp_shard_schedule(H, r, nranks, halo, hy, mode)
+    y0, sh = sc["y0"], sc["strip_h"]
+    buf = np.full((sh + 2 * halo, W), fill, dtype=img.dtype)
+    buf[halo:halo + sh] = img[y0:y0 + sh]
+    for kind, peer, row, n in sc["ops"]:        # emulate the NCCL receives
+        if kind == 1:
+            g0 = y0 - halo + row
+            buf[row:row + n] = img[[(g0 + k) % H for k in range(n)]]
+    return y0, sh, local_call(dev(buf))
+
+
+@pytest.mark.parametrize("nranks", [2, 3, 5, 8])
+@pytest.mark.parametrize("m", [3, 5, 7, 9])
+def test_strips_isp_f32(isp, nranks, m):
+    """Strip launches (RowRange, t_real / b_real = 0 at strip edges) of every rank on a
+    2052-wide image run non-degenerate ISP bodies and reproduce the single-image result
+    bitwise, with the halo rows filled as the NCCL schedule fills them."""
+    H, W = 203, 2052
+    img = synth.uniform_f32(H, W, 77)
+    mask = np.random.default_rng(m).random((m, m)).astype(np.float32)
+    hy = m // 2
+    halo = hy + 1
+    full = dev(img)
+    for mode in MODES:
+        for v in ["tma", "warp", "naive"]:
+            ref = host(isp.isp_filter_ex(full, mask, mode, 0.25, variant=v))
+            got = np.full((H, W), np.nan, dtype=np.float32)
+            for r in range(nranks):
+                isp.isp_clear_plans()
+                y0, sh, out = _strip_run(
+                    isp, img, H, W, halo, hy, nranks, r, mode, np.nan,
+                    lambda b: isp.isp_shard_filter_local_f32(b, H, halo, r, nranks, mask, mode, 0.25, variant=v))
+                got[y0:y0 + sh] = host(out)
+                main = isp.isp_recent_plans()[0]          # launch 0: the rows needing no halo
+                assert not main["degenerate"], (mode, v, r, main)
+                if m != 9 or v != "tma":
+                    assert main["choice"] == CODE[v], (mode, v, r, main)
+            np.testing.assert_array_equal(got, ref, err_msg=f"{mode} {v} P={nranks}")
+
+
+@pytest.mark.parametrize("nranks", [2, 4, 8])
+@pytest.mark.parametrize("m", [3, 5])
+def test_strips_isp_u8(isp, nranks, m):
+    """isp_shard_filter_local_u8: u8 Gaussian strips equal the oracle exactly."""
+    H, W = 150, 2064
+    img = synth.uniform_u8(H, W, 78)
+    mask, div = oracle.gaussian_u8_mask(m)
+    halo = m // 2 + 1
+    for mode in MODES:
+        ref = oracle.filter_u8(img, mask, div, mode, 9)
+        for v in ["warp", "tma", "naive"]:
+            got = np.zeros((H, W), dtype=np.uint8)
+            for r in range(nranks):
+                isp.isp_clear_plans()
+                y0, sh, out = _strip_run(
+                    isp, img, H, W, halo, m // 2, nranks, r, mode, 0,
+                    lambda b: isp.isp_shard_filter_local_u8(b, H, halo, r, nranks, mask, div, mode, 9, variant=v))
+                got[y0:y0 + sh] = host(out)
+                main = isp.isp_recent_plans()[0]
+                assert not main["degenerate"] and main["choice"] == CODE[v], (mode, v, r, main)
+            np.testing.assert_array_equal(got, ref, err_msg=f"{mode} {v} P={nranks}")
+
+
+# ---------------------------------------------------------------- Harris exactness at the threshold
+def _harris_r25(dx, dy, mode, c, y, x):
+    """Exact R25 at (y, x) in Python integers through the oracle's border map."""
+    h, w = dx.shape
+    wts = [1, 2, 1]
+    sxx = syy = sxy = 0
+    for j in range(3):
+        for i in range(3):
+            yy = oracle.border_index(mode, y + j - 1, h)
+            xx = oracle.border_index(mode, x + i - 1, w)
+            if yy < 0 or xx < 0:
+                gx = gy = c
+            else:
+                gx, gy = int(dx[yy, xx]), int(dy[yy, xx])
+            wt = wts[j] * wts[i]
+            sxx += wt * gx * gx
+            syy += wt * gy * gy
+            sxy += wt * gx * gy
+    return 25 * (sxx * syy - sxy * sxy) - (sxx + syy) ** 2
+
+
+def test_harris_threshold_boundary(isp):
+    """thr = R-1, R, R+1 around the true response of chosen pixels (large |R| ~ 1e15,
+    derivatives near +-1020): the f32 sums / f64 response decide exactly as int64."""
+    h, w = 40, 2064
+    rng = np.random.default_rng(123)
+    dx = rng.integers(-1020, 1021, (h, w)).astype(np.int16)
+    dy = rng.integers(-1020, 1021, (h, w)).astype(np.int16)
+    dx[:, ::7] = 1020
+    dy[::5, :] = -1020
+    ddx, ddy = dev(dx), dev(dy)
+    picks = [(0, 0), (h - 1, w - 1), (17, 1030), (3, 700), (39, 5)]
+    for mode in MODES:
+        c = -1020 if mode == "constant" else 0
+        for (y, x) in picks:
+            R = _harris_r25(dx, dy, mode, c, y, x)
+            for thr, want in ((R - 1, 255), (R, 0), (R + 1, 0)):
+                ref = oracle.harris(dx, dy, mode, c, thr)
+                assert ref[y, x] == want
+                for v in ["tma", "warp", "naive"]:
+                    got = host(isp.isp_harris_u8(ddx, ddy, mode, c, thr, variant=v))
+                    ran(isp, v)
+                    assert got[y, x] == want, (mode, v, y, x, thr)
+                    np.testing.assert_array_equal(got, ref, err_msg=f"{mode} {v} thr={thr}")
+
+
+def test_harris_const_range(isp):
+    d = dev(np.zeros((8, 16), dtype=np.int16))
+    with pytest.raises(isp.IspError):
+        isp.isp_harris_u8(d, d, "constant", 1021, 0)
+    with pytest.raises(isp.IspError):
+        isp.isp_harris_u8(d, d, "constant", -1021, 0)
+
+
+# ---------------------------------------------------------------- Sobel magnitude near ties
+def _sobel_block(X, Y, rng):
+    """A 3x3 u8 block whose centre Sobel derivatives are exactly (X, Y) (a9: dx = (c-a) +
+    2(f-d) + (i-g), dy = (g-a) + 2(h-b) + (i-c) over [[a,b,c],[d,e,f],[g,h,i]])."""
+    for _ in range(200000):
+        a, c, g, i = (int(t) for t in rng.integers(0, 256, 4))
+        r1, r2 = X - (c - a) - (i - g), Y - (g - a) - (i - c)
+        if r1 % 2 or r2 % 2 or abs(r1 // 2) > 255 or abs(r2 // 2) > 255:
+            continue
+        fd, hb = r1 // 2, r2 // 2
+        d_, b_ = max(0, -fd), max(0, -hb)
+        f_, h_ = d_ + fd, b_ + hb
+        blk = np.array([[a, b_, c], [d_, 128, f_], [g, h_, i]])
+        if blk.min() >= 0 and blk.max() <= 255:
+            return blk.astype(np.uint8)
+    raise AssertionError((X, Y))
+
+
+def test_sobel_magnitude_near_ties(isp):
+    """Magnitude rounding next to every half-integer: n = dx^2 + dy^2 within +-4 of
+    (k + 1/2)^2 = k^2 + k + 1/4 for k = 1..255 (the tightest margins of the sqrt.approx
+    rounding: 0.25/(2k+1) at n = k^2 + k).  Sobel
+    derivatives of u8 images satisfy dx = dy (mod 2) (dx + dy = 2(i - a) + even terms),
+    so only n = 0 (mod 4) or 2 (mod 8) occur: the test places every reachable n of the
+    band, with both signs, at centres of isolated 3x3 blocks and compares the whole
+    image with the oracle."""
+    targets = []
+    for k in range(1, 256):
+        for n in range(k * k + k - 4, k * k + k + 5):
+            for X in range(0, 257):
+                r = n - X * X
+                if r < 0:
+                    break
+                Y = int(round(r ** 0.5))
+                if Y * Y == r and (X - Y) % 2 == 0:
+                    sx, sy = (1, -1)[len(targets) % 2], (1, -1)[(len(targets) // 2) % 2]
+                    targets.append((sx * X, sy * Y, n))
+                    break
+    assert len(targets) >= 150
+    rng = np.random.default_rng(5)
+    nb = len(targets)
+    per_row = 680
+    rows = -(-nb // per_row)
+    img = np.zeros((3 * rows + 6, 3 * per_row + 24), dtype=np.uint8)   # 2064 wide: 16-B aligned rows
+    centres = []
+    for t, (X, Y, n) in enumerate(targets):
+        by, bx = 3 + 3 * (t // per_row), 3 * (t % per_row)
+        img[by:by + 3, bx:bx + 3] = _sobel_block(X, Y, rng)
+        centres.append((by + 1, bx + 1, X, Y, n))
+    d = dev(img)
+    for mode in MODES:
+        rdx, rdy, rmag = oracle.sobel(img, mode, 0)
+        for (y, x, X, Y, n) in centres:
+            assert int(rdx[y, x]) ** 2 + int(rdy[y, x]) ** 2 == n
+        for v in ["tma", "warp", "naive"]:
+            dx, dy, mag = isp.isp_sobel_u8(d, mode, 0, variant=v)
+            ran(isp, v)
+            np.testing.assert_array_equal(host(mag), rmag, err_msg=f"{mode} {v}")

@@ -7,9 +7,11 @@ Bars (BASELINE.json north_star):
     (reading A28; the oracle accumulates in double);
   * Bilateral: max-abs <= 1e-4 on [0,1] data;
   * ISP_BLOCK, ISP_WARP, ISP_AUTO results are bitwise identical to ISP_NAIVE.
-Sizes: several tiles plus ragged tails (odd widths/heights), degenerate plans (windows
-larger than the image), misaligned bases/pitches, and BASELINE.json's full sizes on
-sampled rows in the launch configuration bench.py times.
+Sizes here: the FALLBACK shapes -- odd / misaligned widths (the planner sends them to
+the naive kernel, which must still equal the oracle), tiny and degenerate plans (windows
+larger than the image, reading A3) -- and BASELINE.json's full sizes on sampled rows in
+the launch configuration bench.py times.  The aligned multi-tile shapes that run every
+ISP region body (with the plan asserted) are in test_gpu_isp_bodies.py.
 """
 import numpy as np
 import pytest
@@ -55,6 +57,7 @@ def binomial_f32(m):
     return (np.outer(b, b) / b.sum() ** 2).astype(np.float32)
 
 
+# fallback shapes: misaligned widths (naive kernel) and tiny / degenerate plans
 SHAPES = [(1, 1), (3, 5), (64, 64), (37, 517), (130, 1001), (257, 1031)]
 
 
@@ -229,7 +232,7 @@ def test_atrous(isp, shape, d):
         ref = oracle.atrous(img, d, mode, 0.75)
         outs = [host(isp.isp_atrous_f32(t, d, mode, 0.75, variant=v)) for v in VARIANTS]
         for o in outs:
-            check_f32(o, ref, np.maximum(np.abs(ref), 0.75))
+            check_f32(o, ref, np.abs(ref))        # A28: non-negative weights and data => scale |o|
             np.testing.assert_array_equal(o, outs[-1])
 
 
@@ -238,7 +241,7 @@ def test_night(isp):
     for mode in MODES:
         ref = oracle.night(img, mode, 0.25)
         got = host(isp.isp_night_f32(dev(img), mode, 0.25))
-        check_f32(got, ref, np.abs(ref), tol=2e-6 * 5)
+        check_f32(got, ref, np.abs(ref), tol=4e-5)   # 4 passes x A28 (see test_night_bodies)
 
 
 # ---------------------------------------------------------------- BASELINE.json configs, full size
@@ -327,9 +330,9 @@ def test_cfg5_gauss7_f32_16384_single_gpu(isp):
 @pytest.mark.parametrize("nranks", [2, 3, 5, 8])
 @pytest.mark.parametrize("m", [3, 5, 7, 9])
 def test_strips_local_equal_full_image(isp, nranks, m):
-    """The strip launches of every rank (isp_shard_filter_local_f32: RowRange, t_real /
-    b_real, halo clamping) with halos filled exactly as the NCCL schedule fills them
-    (neighbour rows; ring wrap for Repeat) reproduce the single-image result bitwise."""
+    """Fallback strips: W = 333 is narrower than one ISP tile, so every strip launch is a
+    degenerate plan (NAIVE); the strip/halo plumbing must still reproduce the
+    single-image result bitwise.  The ISP strip bodies: test_gpu_isp_bodies.py."""
     H, W = 203, 333
     img = synth.uniform_f32(H, W, 77)
     mask = np.random.default_rng(m).random((m, m)).astype(np.float32)
