@@ -61,18 +61,32 @@ def peaks():
         return {}
 
 
-def ncu_traffic():
-    """Per-launch DRAM bytes (read + write) of the dominant kernel from the newest committed
-    `ncu --set full` summary (profiles/r<NN>_ncu_summary.json, tools/ncu_summary.py)."""
-    import glob
-    paths = sorted(glob.glob(os.path.join(ROOT, "profiles", "r*_ncu_summary.json")))
-    if not paths:
+def lib_digest():
+    import hashlib
+    try:
+        h = hashlib.sha256(open(os.path.join(ROOT, "paper_conf_ipps_qiaoth21_b200", "libisp.so"), "rb").read())
+        return h.hexdigest()[:16]
+    except OSError:
         return None
+
+
+def ncu_traffic(workload):
+    """DRAM bytes (read + write) per launch of the dominant kernel, measured by ncu over a
+    range of >= 8 back-to-back launches (so write-backs are counted) -- `ncu` replays
+    kernels, so it cannot run inside this timed process; tools/ncu_traffic.py writes
+    profiles/r<NN>_traffic_<workload>.json and records the libisp.so digest it measured.
+    Returned with its source file and whether that digest matches the library loaded now."""
+    import glob
+    paths = sorted(glob.glob(os.path.join(ROOT, "profiles", f"r*_traffic_{workload}.json")))
+    if not paths:
+        return {"traffic": None, "traffic_source": None}
     try:
         d = json.load(open(paths[-1]))
-        return d.get("dominant_kernel", {}).get("dram_bytes_per_launch")
     except Exception:
-        return None
+        return {"traffic": None, "traffic_source": None}
+    return {"traffic": d.get("dram_bytes_per_launch"), "traffic_source": os.path.relpath(paths[-1], ROOT),
+            "traffic_build_matches": d.get("libisp_sha16") == lib_digest(),
+            "traffic_launches": d.get("launches")}
 
 
 class ClockSampler:
@@ -138,39 +152,44 @@ def cpu_model():
     return platform.processor() or "unknown"
 
 
-def _oracle_rows_rate(img, mask, threads, target_s):
+def _oracle_rows_rate(img, mask, modes, threads, target_s):
     """Oracle throughput (Mpixel/s) on a centred row band sized for ~target_s seconds."""
     import oracle
+    H, W = img.shape
     t = time.perf_counter()
-    for m in MODES:
+    for m in modes:
         oracle.filter_f64(img, mask, m, CONST, rows=(0, 2 * threads), threads=threads)
     dt = time.perf_counter() - t
-    rows = int(max(threads, min(N_SIDE, 2 * threads * target_s / max(dt, 1e-6))))
+    rows = int(max(threads, min(H, 2 * threads * target_s / max(dt, 1e-6))))
     rows -= rows % threads
     rows = max(rows, threads)
-    y0 = (N_SIDE - rows) // 2
+    y0 = (H - rows) // 2
     t = time.perf_counter()
-    for m in MODES:
+    for m in modes:
         oracle.filter_f64(img, mask, m, CONST, rows=(y0, y0 + rows), threads=threads)
     dt = time.perf_counter() - t
-    px = 4 * rows * N_SIDE
-    return px / dt / 1e6, f"rows [{y0},{y0 + rows}) x 4 modes ({px} px, {dt:.1f} s)", dt
+    px = len(modes) * rows * W
+    return px / dt / 1e6, f"rows [{y0},{y0 + rows}) x {len(modes)} modes ({px} px, {dt:.1f} s)", dt
 
 
-def cpu_oracle_rate(target_s=8.0, threads=None):
+def cpu_oracle_rate(target_s=8.0, threads=None, workload=None):
     """Oracle (oracle/ C, double accumulation, per-read border map) on the host cores over a
-    bounded row sample of the same workload, all four modes: once on 1 thread and once on
-    all cores.  `value` / `cores` are the all-core run."""
+    bounded row sample of the same workload and modes: once on 1 thread and once on all
+    cores.  `value` / `cores` are the all-core run."""
     import oracle
     import synth
     threads = threads or os.cpu_count() or 1
     oracle.build_oracle()
-    img = synth.uniform_f32(N_SIDE, N_SIDE, synth.CONFIG_SEEDS["cfg2"])
-    mask = gauss_mask()
-    v1, s1, d1 = _oracle_rows_rate(img, mask, 1, target_s / 2)
-    vn, sn, dn = _oracle_rows_rate(img, mask, threads, target_s)
+    if workload is None or workload.name == "cfg2":
+        img = synth.uniform_f32(N_SIDE, N_SIDE, synth.CONFIG_SEEDS["cfg2"])
+        mask, modes, name = gauss_mask(), MODES, "cfg2 4096x4096"
+    else:   # cfg5: a 512-row band of the 16384-wide image is enough for the bounded sample
+        img = synth.uniform_f32(512, workload.W, synth.CONFIG_SEEDS["cfg5"])
+        mask, modes, name = workload.mask(), workload.modes, "cfg5 16384-wide (512-row band)"
+    v1, s1, d1 = _oracle_rows_rate(img, mask, modes, 1, target_s / 2)
+    vn, sn, dn = _oracle_rows_rate(img, mask, modes, threads, target_s)
     return {"value": vn, "unit": UNIT, "cores": threads, "kind": "oracle",
-            "sample": f"cfg2 4096x4096 image, all cores: {sn}; 1 thread: {s1}",
+            "sample": f"{name} image, all cores: {sn}; 1 thread: {s1}",
             "single_thread": {"value": v1, "unit": UNIT, "cores": 1, "sample": s1, "seconds": d1},
             "cpu_model": cpu_model(), "seconds": dn + d1}
 
@@ -212,6 +231,34 @@ def run_reference(args):
 
 
 # ------------------------------------------------------------------------------------------
+class Workload:
+    """cfg2 (default, BASELINE.json configs[1]): 5x5 binomial f32, 4 border modes, 4096^2
+    per rank -- N ranks = row strips of a (4096 N) x 4096 image (weak scaling).
+    cfg5 (configs[4], the north-star scaling case): 7x7 binomial f32 on ONE 16384^2 image,
+    Clamp and Repeat, row strips over N ranks (strong scaling)."""
+
+    def __init__(self, name, world):
+        self.name = name
+        if name == "cfg2":
+            self.W, self.H = N_SIDE, N_SIDE * world
+            self.window, self.modes, self.scaling = WINDOW, MODES, "weak"
+            self.seed = 2
+            self.desc = ("cfg2: 5x5 binomial Gaussian f32 4096x4096 per rank, 4 border modes "
+                         "(clamp, mirror, repeat, constant), variant auto (isp+m)")
+        else:
+            self.W = self.H = 16384
+            self.window, self.modes, self.scaling = 7, ["clamp", "repeat"], "strong"
+            self.seed = 5
+            self.desc = ("cfg5: 7x7 binomial Gaussian f32 on one 16384x16384 image, clamp + repeat, "
+                         "variant auto (isp+m)")
+        self.halo = self.window // 2
+
+    def mask(self):
+        import synth
+        b = synth.binomial_row(self.window).astype(np.float64)
+        return (np.outer(b, b) / b.sum() ** 2).astype(np.float32)
+
+
 def run_isp(args):
     import torch
     import torch.distributed as dist
@@ -225,20 +272,32 @@ def run_isp(args):
     if world > 1:
         dist.init_process_group("nccl", device_id=dev)
     isp.lib()
-    mask = gauss_mask()
-    H_img = N_SIDE * world
-    halo = WINDOW // 2
-    # ---- inputs: the seeded cfg2 image (rank r: its strip of the tall image) ----
-    host_img = synth.uniform_f32(N_SIDE, N_SIDE, synth.CONFIG_SEEDS["cfg2"] + rank)
+    wl = Workload(args.workload, world)
+    mask = wl.mask()
+    modes = wl.modes
+    nm = len(modes)
+    H_img, W = wl.H, wl.W
+    halo = wl.halo
+    y0, sh = isp.isp_shard_rows(H_img, rank, world) if world > 1 else (0, H_img)
+    # ---- inputs: seeded, resident in HBM before the timed region ----
+    if wl.name == "cfg2":
+        host_img = synth.uniform_f32(N_SIDE, N_SIDE, synth.CONFIG_SEEDS["cfg2"] + rank)
+        src = torch.from_numpy(host_img)
+    else:
+        g = torch.Generator().manual_seed(wl.seed * 1000 + rank)
+        src = torch.rand((sh, W), generator=g)
+        host_img = None
+    img_bytes = 2 * 4 * sh * W                       # one in + one out buffer
+    npairs = NPAIRS if wl.name == "cfg2" else int(min(6, max(2, -(-2 * 126 * 2 ** 20 // img_bytes))))
     pairs = []
-    for _ in range(NPAIRS):
+    for _ in range(npairs):
         if world > 1:
-            strip = torch.empty((N_SIDE + 2 * halo, N_SIDE), dtype=torch.float32, device=dev)
-            strip[halo:halo + N_SIDE].copy_(torch.from_numpy(host_img))
+            strip = torch.empty((sh + 2 * halo, W), dtype=torch.float32, device=dev)
+            strip[halo:halo + sh].copy_(src)
             inp = strip
         else:
-            inp = torch.from_numpy(host_img).to(dev)
-        out = torch.empty((N_SIDE, N_SIDE), dtype=torch.float32, device=dev)
+            inp = src.to(dev)
+        out = torch.empty((sh, W), dtype=torch.float32, device=dev)
         pairs.append((inp, out))
     ctx = None
     comm_stream = torch.cuda.Stream(device=dev)
@@ -258,19 +317,23 @@ def run_isp(args):
             isp.isp_filter_ex(inp, mask, mode, CONST, out=out, variant=v, stream=stream)
 
     def step(k, v=variant):
-        for i, m in enumerate(MODES):
-            launch(m, (4 * k + i) % NPAIRS, v)
+        for i, m in enumerate(modes):
+            launch(m, (nm * k + i) % npairs, v)
 
-    launches_per_step = 4 * (len([l for l in isp.isp_shard_schedule(H_img, rank, world, halo, halo, 0)["launch"]
-                                  if l[1] > 0]) if world > 1 else 1)
-    nphase = NPAIRS // np.gcd(4, NPAIRS)          # rotation period in steps
+    if world > 1:
+        launches_per_step = sum(len([l for l in isp.isp_shard_schedule(H_img, rank, world, halo, halo,
+                                                                       isp.MODES[m])["launch"] if l[1] > 0])
+                                for m in modes)
+    else:
+        launches_per_step = nm
+    nphase = npairs // int(np.gcd(nm, npairs))      # rotation period in steps
     use_graph = not args.no_graph
 
     with torch.cuda.stream(stream):
         for k in range(max(args.warmup, 1)):      # warm-up (also loads every kernel)
             step(k)
     torch.cuda.synchronize()
-    # The timed region replays ONE graph holding exactly K steps (4K launches back to
+    # The timed region replays ONE graph holding exactly K steps (all launches back to
     # back, no inter-graph gaps); above MAX_GRAPH_STEPS steps it is a chunk graph of
     # MAX_GRAPH_STEPS steps replayed, plus one graph for the remainder.
     MAX_GRAPH_STEPS = 2000
@@ -333,40 +396,44 @@ def run_isp(args):
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         ms = float(t.item())
     clocks = cs.summary(t_wall0, t_wall1)
-    px_step = 4 * N_SIDE * N_SIDE * world
+    px_step = nm * H_img * W                 # output pixels of all ranks per step
     value = px_step * args.steps / (ms / 1e3) / 1e6
     ms_step = ms / args.steps
 
-    # ---- per-launch duration of the dominant kernel (the ISP 5x5 f32 stencil) ----
-    per_launch_us = 1e3 * ms_step / 4.0
+    # ---- per-launch duration of the dominant kernel (the ISP stencil) on this rank ----
+    per_launch_us = 1e3 * ms_step / nm
     pk = peaks()
     hbm = pk.get("hbm_gbs")
-    achieved = BYTES_PER_PX * N_SIDE * N_SIDE / (per_launch_us * 1e-6) / 1e9
+    rank_bytes = BYTES_PER_PX * sh * W
+    achieved = rank_bytes / (per_launch_us * 1e-6) / 1e9
+    kname = f"OpSepF32<{wl.window},{wl.window}>"
     roof = {"bound": "hbm", "achieved": achieved, "peak": hbm if hbm else 6650.0, "unit": "GB/s",
-            "frac": achieved / (hbm if hbm else 6650.0), "traffic": ncu_traffic(),
-            "peak_source": "MEASURED_PEAKS.json hbm_gbs" if hbm else "fallback (B200_PROFILING.md)",
-            "kernel": f"variant {args.variant}: " + ("k_staged<OpSepF32<5,5>> (TMA-staged ISP)" if plan["choice"] == 4 else "k_stencil<OpSepF32<5,5>>"),
-            "algorithmic_bytes_per_launch": BYTES_PER_PX * N_SIDE * N_SIDE,
+            "frac": achieved / (hbm if hbm else 6650.0),
+            "peak_source": "MEASURED_PEAKS.json hbm_gbs (measured)" if hbm else "fallback (B200_PROFILING.md)",
+            "kernel": f"variant {args.variant}: " + (f"k_pstaged<{kname}> (TMA-staged ISP)" if plan["choice"] == 4
+                                                     else f"k_stencil<{kname}>"),
+            "algorithmic_bytes_per_launch": rank_bytes,
             "duration_us": per_launch_us,
             "duration_method": "timed region / launches (one CUDA graph of the K steps, kernels back to back)"}
+    roof.update(ncu_traffic(wl.name))
 
     # ---- ISP vs naive per mode (same methodology, single-GPU variants) ----
     variants = {}
     if world == 1 and not args.quick:
-        for m in MODES:
+        for m in modes:
             variants[m] = {}
             for v in ["auto", "tma", "warp", "block", "naive"]:
-                R = 12
+                R = 12 if wl.name == "cfg2" else 4
                 g = torch.cuda.CUDAGraph()
                 with torch.cuda.stream(stream):
                     for i in range(2):
-                        launch(m, i % NPAIRS, v)
+                        launch(m, i % npairs, v)
                 torch.cuda.synchronize()
                 with torch.cuda.graph(g, stream=stream):
                     for i in range(R):
-                        launch(m, i % NPAIRS, v)
+                        launch(m, i % npairs, v)
                 torch.cuda.synchronize()
-                reps = 40
+                reps = 40 if wl.name == "cfg2" else 5
                 a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
                 with torch.cuda.stream(stream):
                     g.replay()
@@ -376,18 +443,35 @@ def run_isp(args):
                     b.record(stream)
                 torch.cuda.synchronize()
                 us = 1e3 * a.elapsed_time(b) / (reps * R)
-                variants[m][v] = {"us": us, "gbs": BYTES_PER_PX * N_SIDE * N_SIDE / (us * 1e-6) / 1e9,
-                                  "mpix_s": N_SIDE * N_SIDE / us}
-            variants[m]["speedup_tma_vs_naive"] = variants[m]["naive"]["us"] / variants[m]["tma"]["us"]
-            variants[m]["speedup_warp_vs_naive"] = variants[m]["naive"]["us"] / variants[m]["warp"]["us"]
-            variants[m]["speedup_auto_vs_naive"] = variants[m]["naive"]["us"] / variants[m]["auto"]["us"]
+                variants[m][v] = {"us": us, "gbs": BYTES_PER_PX * H_img * W / (us * 1e-6) / 1e9,
+                                  "mpix_s": H_img * W / us}
+            for v in ("tma", "warp", "auto"):
+                variants[m][f"speedup_{v}_vs_naive"] = variants[m]["naive"]["us"] / variants[m][v]["us"]
+
+    # ---- halo exchange alone (N > 1): NCCL send/recv of the strip edges on the comm stream ----
+    halo_us = None
+    if world > 1:
+        inp = pairs[0][0]
+        R = 50
+        dist.barrier()
+        torch.cuda.synchronize()
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        with torch.cuda.stream(comm_stream):
+            a.record(comm_stream)
+            for _ in range(R):
+                isp.isp_shard_exchange(ctx, inp, H_img, halo, halo, modes[-1], comm_stream=comm_stream)
+            b.record(comm_stream)
+        torch.cuda.synchronize()
+        t = torch.tensor([a.elapsed_time(b) * 1e3 / R], device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        halo_us = float(t.item())
 
     # ---- end to end: pinned host buffers, H2D + filter + D2H inside the timed region ----
     e2e = None
     if not args.quick:
-        hin = torch.from_numpy(host_img).pin_memory()
-        houts = [torch.empty((N_SIDE, N_SIDE), dtype=torch.float32).pin_memory() for _ in range(2)]
-        E = max(3, min(20, args.steps // 100))
+        hin = (torch.from_numpy(host_img) if host_img is not None else src).pin_memory()
+        houts = [torch.empty((sh, W), dtype=torch.float32).pin_memory() for _ in range(2)]
+        E = max(3, min(20, args.steps // 100)) if wl.name == "cfg2" else 3
         if world > 1:
             dist.barrier()
         torch.cuda.synchronize()
@@ -395,9 +479,9 @@ def run_isp(args):
         with torch.cuda.stream(stream):
             a.record(stream)
             for k in range(E):
-                for i, m in enumerate(MODES):
-                    inp, out = pairs[i % NPAIRS]
-                    dst = inp[halo:halo + N_SIDE] if world > 1 else inp
+                for i, m in enumerate(modes):
+                    inp, out = pairs[i % npairs]
+                    dst = inp[halo:halo + sh] if world > 1 else inp
                     dst.copy_(hin, non_blocking=True)
                     if world > 1:
                         isp.isp_shard_filter_f32(ctx, inp, H_img, halo, mask, m, CONST, out=out, stream=stream,
@@ -413,40 +497,91 @@ def run_isp(args):
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
             ems = float(t.item())
         e2e = {"value": px_step * E / (ems / 1e3) / 1e6, "unit": UNIT,
-               "h2d_bytes_per_step": 4 * N_SIDE * N_SIDE * 4, "d2h_bytes_per_step": 4 * N_SIDE * N_SIDE * 4,
-               "steps": E, "ms_per_step": ems / E, "api": "isp_filter via the Python binding, pinned host buffers"}
+               "h2d_bytes_per_step": nm * 4 * sh * W, "d2h_bytes_per_step": nm * 4 * sh * W,
+               "steps": E, "ms_per_step": ems / E,
+               "api": "isp_filter / isp_shard_filter_f32 via the Python binding, pinned host buffers"}
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu:
-        cpu = cpu_oracle_rate()
+        cpu = cpu_oracle_rate(workload=wl)
 
     if ctx is not None:
         torch.cuda.synchronize()
         isp.isp_shard_destroy(ctx)
     if rank == 0:
         line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
-                "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True, "scaling": "weak",
+                "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True, "scaling": wl.scaling,
                 "vs_baseline": None, "dtype": "f32", "data": "synthetic",
-                "config": {"workload": "cfg2: 5x5 binomial Gaussian f32 4096x4096 per rank, 4 border modes "
-                                       "(clamp, mirror, repeat, constant), variant auto (isp+m)"
-                                       + (f"; {world} ranks = row strips of a {H_img}x4096 image, NCCL halo exchange"
-                                          if world > 1 else ""),
-                           "image": [H_img, N_SIDE], "window": [WINDOW, WINDOW], "const": CONST,
-                           "l2": f"rotating {NPAIRS} in/out buffer pairs ({NPAIRS * 128} MiB > 2x L2)",
+                "config": {"workload": wl.desc
+                                       + (f"; {world} ranks = row strips of the {H_img}x{W} image, NCCL halo "
+                                          "exchange" if world > 1 else ""),
+                           "image": [H_img, W], "window": [wl.window, wl.window], "const": CONST,
+                           "modes": modes,
+                           "l2": f"rotating {npairs} in/out buffer pairs "
+                                 f"({npairs * img_bytes // 2 ** 20} MiB per rank > 2x L2)",
                            "parallelism": f"row-strips x{world}" if world > 1 else "single GPU",
                            "cuda_graphs": use_graph, "plan": {k: plan[k] for k in
-                                                              ("tile_w", "tile_h", "choice", "g", "degenerate")}},
+                                                              ("tile_w", "tile_h", "nx", "ny", "choice", "g",
+                                                               "degenerate")}},
                 "roofline": roof, "cpu_baseline": cpu, "e2e": e2e,
                 "gpu_launches": args.steps * launches_per_step, "clocks": clocks,
                 "isp_vs_naive": variants or None}
+        if world > 1:
+            line["halo_exchange_us"] = halo_us
+            line["per_rank_rows"] = sh
         print(json.dumps(line), flush=True)
     if world > 1:
         dist.destroy_process_group()
 
 
+def check_launch(args):
+    """--check-launch: the multi-rank launch path without a workload -- every rank joins
+    the process group (NCCL on GPUs, gloo on a CPU box), all-reduces its rank id, rank 0
+    prints what it saw.  Used by tests/test_bench_launch.py on CPU."""
+    import torch
+    import torch.distributed as dist
+    rank, world, local = env_rank()
+    backend = "nccl" if torch.cuda.is_available() else "gloo"
+    if world > 1:
+        if backend == "nccl":
+            torch.cuda.set_device(local)
+            dist.init_process_group(backend, device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group(backend)
+    t = torch.tensor([float(rank)], device="cuda" if backend == "nccl" else "cpu")
+    n = torch.ones(1, device=t.device)
+    if world > 1:
+        dist.all_reduce(t)
+        dist.all_reduce(n)
+    if rank == 0:
+        print(json.dumps({"check": "launch", "world_size": world, "gpus_requested": args.gpus, "backend": backend,
+                          "ranks_seen": int(n.item()), "rank_sum": int(t.item())}), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+def spawn_ranks(args):
+    """`bench.py --gpus N` started without torchrun: re-exec under torch.distributed.run with
+    N ranks on this node (rendezvous on 127.0.0.1), as the driver does."""
+    import socket
+    with socket.socket() as sk:
+        sk.bind(("127.0.0.1", 0))
+        port = sk.getsockname()[1]
+    env = dict(os.environ)
+    env.setdefault("NCCL_DEBUG", "INFO")          # NCCL's init lines (nranks) stay visible
+    env.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+           "--master-addr", "127.0.0.1", f"--master-port={port}", os.path.abspath(__file__)] + sys.argv[1:]
+    return subprocess.call(cmd, env=env)
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--workload", default="cfg2", choices=["cfg2", "cfg5"],
+                    help="cfg2: BASELINE configs[1] (default, weak scaling over ranks); "
+                         "cfg5: configs[4] 16384^2 7x7 strong scaling")
+    ap.add_argument("--check-launch", action="store_true", help="only check the N-rank launch path")
     ap.add_argument("--steps", type=int, default=6000)
     ap.add_argument("--warmup", type=int, default=20)
     ap.add_argument("--impl", default="isp", choices=["isp", "reference"])
@@ -457,6 +592,14 @@ def main():
     args = ap.parse_args()
     if args.warmup < 3:
         ap.error("--warmup must be >= 3")
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        sys.exit(spawn_ranks(args))
+    world = int(os.environ.get("WORLD_SIZE", 1))
+    if world != args.gpus:
+        ap.error(f"--gpus {args.gpus} but WORLD_SIZE={world}")
+    if args.check_launch:
+        check_launch(args)
+        return
     if args.impl == "reference":
         run_reference(args)
     else:

@@ -236,6 +236,11 @@ isp_status_t isp_shard_filter_u8(isp_shard_ctx *ctx, uint8_t *strip, int w, int 
 isp_status_t isp_shard_filter_local_f32(float *strip, int w, int H, int pitch, int halo, int rank, int nranks,
                                         const float *mask, int mw, int mh, int border_mode, float const_val,
                                         float *out, int out_pitch, isp_variant_t variant, isp_stream_t stream);
+/* Only the halo exchange of isp_shard_filter_* (the schedule's NCCL send/recv, rows of
+ * `pitch` elements of `elem_size` bytes) on comm_stream -- for timing the exchange alone
+ * and for callers that run their own launches.  Stream-ordered; no filtering. */
+isp_status_t isp_shard_exchange(isp_shard_ctx *ctx, void *strip, int elem_size, int H, int pitch, int halo, int hy,
+                                int border_mode, isp_stream_t comm_stream);
 /* u8 counterpart of isp_shard_filter_local_f32 (the launch part of isp_shard_filter_u8). */
 isp_status_t isp_shard_filter_local_u8(uint8_t *strip, int w, int H, int pitch, int halo, int rank, int nranks,
                                        const int32_t *mask, int mw, int mh, int32_t divisor, int border_mode,

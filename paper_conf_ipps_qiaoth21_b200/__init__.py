@@ -28,7 +28,7 @@ __all__ = [
     "isp_set_launch_override",
     "isp_shard_unique_id", "isp_shard_init", "isp_shard_rows", "isp_shard_schedule",
     "isp_shard_filter_f32", "isp_shard_filter_u8", "isp_shard_filter_local_f32", "isp_shard_filter_local_u8",
-    "isp_shard_destroy",
+    "isp_shard_exchange", "isp_shard_destroy",
 ]
 
 CLAMP, MIRROR, REPEAT, CONSTANT = 0, 1, 2, 3
@@ -115,6 +115,7 @@ _SIGS = {
     "isp_shard_filter_local_f32": [_P, _I, _I, _I, _I, _I, _I, _P, _I, _I, _I, _F, _P, _I, _I, _P],
     "isp_shard_filter_local_u8": [_P, _I, _I, _I, _I, _I, _I, _P, _I, _I, ctypes.c_int32, _I, _I, _P, _I, _I, _P],
     "isp_recent_plans": [_P, _I],
+    "isp_shard_exchange": [_P, _P, _I, _I, _I, _I, _I, _I, _P],
 }
 
 _lib = None
@@ -495,6 +496,17 @@ def isp_shard_filter_local_u8(strip, H, halo, rank, nranks, mask, divisor, borde
                                            mw, mh, int(divisor), _mode(border_mode), int(const_val), out.data_ptr(),
                                            out.shape[1], _variant(variant), _stream(strip, stream)))
     return out
+
+
+def isp_shard_exchange(ctx, strip, H, halo, hy, border_mode, comm_stream=None, rank=None, nranks=None):
+    """Only the NCCL halo exchange of a strip buffer (include/isp.h)."""
+    if not isinstance(strip, torch.Tensor) or not strip.is_cuda or strip.dim() != 2 or not strip.is_contiguous():
+        raise ValueError("strip must be a contiguous 2-D CUDA tensor")
+    rank, nranks = _ctx_ranks(ctx, rank, nranks)
+    _strip_rows(strip, H, halo, rank, nranks, hy)
+    cs = comm_stream if comm_stream is not None else torch.cuda.current_stream(strip.device)
+    _check(lib().isp_shard_exchange(ctx, strip.data_ptr(), strip.element_size(), int(H), strip.shape[1], int(halo),
+                                    int(hy), _mode(border_mode), ctypes.c_void_p(cs.cuda_stream)))
 
 
 def isp_shard_destroy(ctx):

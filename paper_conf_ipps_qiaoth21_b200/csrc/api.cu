@@ -88,6 +88,10 @@ struct Plan {
     int bh_l, bh_r, bh_t, bh_b, w_l, w_r;
     int edge_w;  // balanced split: weight of the image's first / last strip (x 1/256)
     bool degenerate;
+    // pixel rows of the block rows in the T class (by < BH_T), the middle class and the
+    // B class (by >= BH_B): uniform tiles -> count * ty (Eq. 5 as printed, reading A25);
+    // balanced split -> the real rows of those block rows
+    long long rows_t, rows_m, rows_b;
 };
 
 int g_num_sms = 0;
@@ -175,6 +179,16 @@ Plan make_plan(int w, int h, int hx, int hy, int px, int tile_w_req, int tile_h_
             while (bb > 0 && y0_of(bb) + hy > h) --bb;   // y0_of(bb) = end of block bb-1
         p.bh_t = bt;
         p.bh_b = bb;
+        if (bt <= bb) {
+            p.rows_t = y0_of(bt) - y0_of(0);
+            p.rows_m = y0_of(bb) - y0_of(bt);
+            p.rows_b = y0_of(p.ny) - y0_of(bb);
+        }
+    }
+    if (p.ty > 0 && p.bh_t <= p.bh_b) {
+        p.rows_t = (long long)p.bh_t * p.ty;
+        p.rows_m = (long long)(p.bh_b - p.bh_t) * p.ty;
+        p.rows_b = (long long)(p.ny - p.bh_b) * p.ty;
     }
     p.degenerate = p.bh_l > p.bh_r || p.bh_t > p.bh_b;
     return p;
@@ -200,6 +214,16 @@ void n_block(const Plan &p, long long nb[9])
 const int kNSwitch[9] = {2, 3, 3, 6, 8, 8, 8, 9, 8};
 
 // Eqs. (3)-(6), (9), (10).
+// Eqs. (3)-(6), (9), (10).  h: rows of the launch's iteration space (the whole image, or a
+// strip's rows).  Regions are products of a column class (L: bx < BH_L, middle, R) and a
+// row class (T, middle, B); the pixels of region r are ncols(r) * tile_w * rows(class),
+// which is n_block(r) * tx * ty for uniform tiles (Eq. 5) and the real block rows for the
+// balanced split.  Forms (reading A14 / A21):
+//   T (0): n(r) = n_switch(r) threads n_block(r) + n_region(r) m n pixels(r)
+//   P (1): n(r) = (n_switch(r) + n_region(r)) m n pixels(r)                     (as printed)
+//   S (2): staged kernels, checks paid per STAGED element E(r) = ncols(r) (tx + 2 hx)
+//          (rows(class) + 2 hy nblockrows(class)):
+//          n(r) = n_switch(r) threads n_block(r) + n_chk(r) n_check E(r) + n_kernel m n pixels(r)
 void model(const Plan &p, int w, int h, int mw, int mh, const isp_model_params &mp, isp_plan_info &o)
 {
     const double m = mw, n = mh, c = mp.n_check, k = mp.n_kernel;
@@ -210,14 +234,28 @@ void model(const Plan &p, int w, int h, int mw, int mh, const isp_model_params &
         o.g = 0;
         return;
     }
-    const double threads = 32.0 * p.wx, pix = (double)p.tile_w * p.ty;
+    const double threads = 32.0 * p.wx, tx = p.tile_w;
+    const double cols[3] = {(double)p.bh_l, (double)(p.bh_r - p.bh_l), (double)(p.nx - p.bh_r)};  // L, mid, R
+    const double rows[3] = {(double)p.rows_t, (double)p.rows_m, (double)p.rows_b};                 // T, mid, B
+    const double brows[3] = {(double)p.bh_t, (double)(p.bh_b - p.bh_t), (double)(p.ny - p.bh_b)};
+    const int hx = mw / 2, hy = mh / 2;
+    // region id (Eq. 4 order) of (row class, column class)
+    static const int kReg[3][3] = {{RG_TL, RG_T, RG_TR}, {RG_L, RG_BODY, RG_R}, {RG_BL, RG_B, RG_BR}};
     double nisp = 0;
-    for (int r = 0; r < 9; ++r) {
-        const double nreg = (r == 0 || r == 1 || r == 3 || r == 4) ? 2 * c + k : (r == 8 ? k : c + k);
-        const double nsw = kNSwitch[r] * mp.ipc_switch;
-        if (mp.form == 1) nisp += (nsw + nreg) * m * n * (double)o.n_block[r] * pix;          // printed
-        else nisp += (nsw * threads + nreg * m * n * pix) * (double)o.n_block[r];             // A14 form T
-    }
+    for (int rc = 0; rc < 3; ++rc)
+        for (int cc = 0; cc < 3; ++cc) {
+            const int r = kReg[rc][cc];
+            const int nchk = (rc != 1) + (cc != 1);                 // Eq. (6), reading A15
+            const double nreg = nchk * c + k;
+            const double nsw = kNSwitch[r] * mp.ipc_switch;
+            const double nb = cols[cc] * brows[rc];
+            const double pix = cols[cc] * tx * rows[rc];
+            if (mp.form == 1) nisp += (nsw + nreg) * m * n * pix;
+            else if (mp.form == 2) {
+                const double E = cols[cc] * (tx + 2.0 * hx) * (rows[rc] + 2.0 * hy * brows[rc]);
+                nisp += nsw * threads * nb + nchk * c * E + k * m * n * pix;
+            } else nisp += nsw * threads * nb + nreg * m * n * pix;
+        }
     o.n_isp = nisp;
     o.r_reduced = o.n_naive / nisp;                                  // Eq. (9)
     o.g = o.r_reduced * o.o_isp / o.o_naive;                         // Eq. (10)
@@ -286,14 +324,42 @@ using RunFn = cudaError_t (*)(const Desc &);
 // 128*PX, halo rounded up to 16 B (HXA) and Eq. (2)'s x bounds taken with HXA and the
 // 16-B aligned width w_al, so every Body CTA's bulk copies are in bounds (A21).
 struct StagedGeom {
-    int hxa, w_al, sw, stages, rs;
+    int hxa, w_al, sw, stages, rs, tail;
     size_t smem;
 };
 
-StagedGeom staged_geom(int w, int hx, int hy, int px, int esz, int nin)
+// Persistent TMA-staged kernel (isp_pstaged.cuh) knobs: compute warps per CTA, unit
+// height CH, ring bytes per CTA, CTAs per SM.
+struct PKnobs {
+    bool on;
+    int nwc, ch, ring_kb, ctas;
+};
+
+int env_int(const char *name, int dflt, int lo, int hi)
+{
+    const char *e = getenv(name);
+    if (!e) return dflt;
+    return std::max(lo, std::min(hi, atoi(e)));
+}
+
+PKnobs pknobs()
+{
+    PKnobs k;
+    // the one-wave static split is the default (measured faster on B200);
+    // ISP_TMA_PERSIST=1 selects the persistent dynamic-unit kernel
+    k.on = env_int("ISP_TMA_PERSIST", 0, 0, 1) == 1 && env_int("ISP_TMA_STATIC", 0, 0, 1) == 0;
+    k.nwc = env_int("ISP_P_NWC", 8, 1, kPMaxComputeWarps);   // best measured: 8 warps x 4 CTAs/SM
+    k.ch = env_int("ISP_P_CH", 16, 1, 4096);
+    k.ring_kb = env_int("ISP_P_RING_KB", 48, 4, 220);
+    k.ctas = env_int("ISP_P_CTAS", 4, 1, 8);
+    return k;
+}
+
+StagedGeom staged_geom(int w, int hx, int hy, int px, int esz, int nin, int nwc = STAGED_WARPS,
+                       bool persistent = false, int ring_kb = 0)
 {
     StagedGeom sg{};
-    const int tw = STAGED_WARPS * 32 * px;
+    const int tw = nwc * 32 * px;
     // halo rounded up to a whole number of 32-B L2 sectors: the bulk copies then start
     // and end on sector boundaries (16-B-aligned copies straddle sectors)
     int align = 32;
@@ -301,29 +367,64 @@ StagedGeom staged_geom(int w, int hx, int hy, int px, int esz, int nin)
     sg.hxa = (int)(ceil_div((long long)hx * esz, align) * align / esz);
     sg.w_al = (int)(((long long)w * esz / 16) * 16 / esz);
     sg.sw = tw + 2 * sg.hxa;
-    // ring of single-row slots, >= 4 slots / ~8 KB of rows in flight per CTA: measured
-    // best on B200 (knobs ISP_RS, ISP_STAGES)
     const long long row_bytes = (long long)nin * sg.sw * esz;
+    if (persistent) {
+        // one row per slot; as many slots as fit the ring budget (>= 4, <= 64)
+        sg.rs = 1;
+        sg.stages = (int)std::min<long long>(kPMaxStages, std::max<long long>(4, (ring_kb * 1024LL) / row_bytes));
+        if (const char *e = getenv("ISP_STAGES")) sg.stages = std::max(2, std::min(kPMaxStages, atoi(e)));
+        sg.smem = kPHeaderBytes + (size_t)sg.stages * row_bytes;
+        return sg;
+    }
+    // ring of single-row slots, >= 4 slots / ~8 KB of rows in flight per CTA: measured
+    // best on B200 for the one-wave static split
     sg.rs = 1;
     if (const char *e = getenv("ISP_RS")) sg.rs = std::max(1, std::min(16, atoi(e)));
     const long long slot_bytes = row_bytes * sg.rs;
     sg.stages = (int)std::min<long long>(32, std::max<long long>(4, ceil_div(8 * 1024, slot_bytes)));
     if (const char *e = getenv("ISP_STAGES")) sg.stages = std::max(2, std::min(32, atoi(e)));
-    sg.smem = 512 + (size_t)sg.stages * slot_bytes;
+    sg.tail = env_int("ISP_TAIL", 1, 0, 1);
+    sg.smem = 640 + (size_t)sg.stages * slot_bytes + (sg.tail ? (size_t)2 * hy * row_bytes : 0);
     return sg;
 }
 
-void apply_staged_bounds(Plan &p, int w, int px, const StagedGeom &sg)
+void apply_staged_bounds(Plan &p, int w, int px, const StagedGeom &sg, int nwc = STAGED_WARPS)
 {
-    p.wx = STAGED_WARPS;
+    p.wx = nwc;
     p.warp_w = 32 * px;
-    p.tile_w = STAGED_WARPS * 32 * px;
+    p.tile_w = nwc * 32 * px;
     p.nx = (int)ceil_div(w, p.tile_w);
     p.bh_l = (int)ceil_div(sg.hxa, p.tile_w);
     p.bh_r = (int)floor_div(sg.w_al - sg.hxa, p.tile_w);
-    p.w_l = p.bh_l * STAGED_WARPS;
-    p.w_r = p.bh_r * STAGED_WARPS;
+    p.w_l = p.bh_l * nwc;
+    p.w_r = p.bh_r * nwc;
     p.degenerate = p.bh_l > p.bh_r || p.bh_t > p.bh_b;
+}
+
+// Scheduler counter pairs of the persistent staged kernels: one pair per (device,
+// stream), 32 B apart, zero between launches (the last CTA of a launch resets its pair).
+unsigned int *sched_counter(cudaStream_t st)
+{
+    static std::mutex mu;
+    static std::unordered_map<int, unsigned int *> pools;
+    static std::unordered_map<long long, int> slots;
+    constexpr int kSlots = 1024;
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess) return nullptr;
+    std::lock_guard<std::mutex> lk(mu);
+    unsigned int *&pool = pools[dev];
+    if (!pool) {
+        if (cudaMalloc(&pool, kSlots * 32) != cudaSuccess || cudaMemset(pool, 0, kSlots * 32) != cudaSuccess ||
+            cudaDeviceSynchronize() != cudaSuccess) {
+            cudaGetLastError();
+            pool = nullptr;
+            return nullptr;
+        }
+    }
+    const long long key = ((long long)dev << 56) ^ (long long)(uintptr_t)st;
+    auto it = slots.find(key);
+    if (it == slots.end()) it = slots.emplace(key, (int)(slots.size() % kSlots)).first;
+    return pool + 8 * it->second;
 }
 
 // Diagnostics: per-CTA timestamps of TMA-staged launches (env ISP_CTA_TRACE), 4 words
@@ -359,17 +460,25 @@ isp_status_t resolve_and_launch(Desc &d, int fam, int w, int h, int mw, int mh, 
         q.disp = disp;
         return kfn(q);
     };
-    const StagedGeom sg = staged_geom(w, hx, hy, px, esz, nin);
-    // runtime-window (direct) ops: the staged variant is the shared-memory tiled kernel
+    // TMA-staged family: persistent dynamic-unit kernel (default) or the one-wave static
+    // split (ISP_TMA_STATIC=1); runtime-window (direct) ops: the shared-memory tiled kernel
     // (isp_direct.cuh k_tile), which needs no alignment
+    const PKnobs pk = pknobs();
+    const bool persist = !direct && pk.on;
+    unsigned int *sched = persist ? sched_counter(d.stream) : nullptr;
+    const bool use_p = persist && sched != nullptr;
+    const int tma_disp = (!direct && !use_p) ? DISP_TMA_STATIC : DISP_TMA;
+    const int nwc = use_p ? pk.nwc : STAGED_WARPS;
+    const StagedGeom sg = staged_geom(w, hx, hy, px, esz, nin, nwc, use_p, pk.ring_kb);
     if (direct) tma_ok = true;
-    tma_ok = tma_ok && fn_of(DISP_TMA) != nullptr && g_override_wx == 0;
-    const int tma_threads = direct ? TILE_THREADS : STAGED_THREADS;
+    tma_ok = tma_ok && fn_of(tma_disp) != nullptr && g_override_wx == 0;
+    const int tma_threads = direct ? TILE_THREADS : 32 * (nwc + 1);
     const size_t tma_smem = direct ? (size_t)(TILE_PX * 32 + 2 * hx) * (TILE_H + 2 * hy) * esz : sg.smem;
     const int nb_naive = blocks_per_sm(fn_of(naive_disp), threads);
     const int nb_stream = blocks_per_sm(fn_of(p0.wx > 1 ? DISP_WARP : DISP_BLOCK), threads);
-    int nb_tma = tma_ok ? blocks_per_sm(fn_of(DISP_TMA), tma_threads, tma_smem) : 0;
+    int nb_tma = tma_ok ? blocks_per_sm(fn_of(tma_disp), tma_threads, tma_smem) : 0;
     if (const char *e = getenv("ISP_CTAS_PER_SM")) nb_tma = std::min(nb_tma, std::max(1, atoi(e)));
+    if (use_p) nb_tma = std::min(nb_tma, pk.ctas);
     if (tma_ok && nb_tma <= 0) tma_ok = false;
 
     isp_variant_t chosen = v;
@@ -382,8 +491,17 @@ isp_status_t resolve_and_launch(Desc &d, int fam, int w, int h, int mw, int mh, 
         if (c == ISP_TMA && direct)  // tiles of TILE_PX*32 x TILE_H, Eq. (2) verbatim
             return make_plan(w, h, hx, hy, px, TILE_PX * 32, TILE_H, TILE_PX * 32, rr, nb_tma);
         if (c == ISP_TMA) {
-            Plan q = make_plan(w, h, hx, hy, px, STAGED_WARPS * 32 * px, 0, 0, rr, nb_tma);
-            apply_staged_bounds(q, w, px, sg);
+            // persistent: uniform tiles of nwc*32*px x CH (Eq. 2 verbatim in y);
+            // static: the balanced one-wave row split
+            int ch = use_p ? pk.ch : 0;
+            if (use_p) {
+                // short launches: halve the unit height until every resident CTA gets a
+                // unit (load balance) -- also keeps Eq. (2) non-degenerate in y
+                const long long nxu = ceil_div(w, (long long)nwc * 32 * px), nrw = rr ? rr->nrows : h;
+                while (ch > 1 && nxu * ceil_div(nrw, ch) < (long long)num_sms() * nb_tma) ch /= 2;
+            }
+            Plan q = make_plan(w, h, hx, hy, px, nwc * 32 * px, ch, 0, rr, nb_tma);
+            apply_staged_bounds(q, w, px, sg, nwc);
             return q;
         }
         // streaming / naive kernels: uniform tiles of kStreamTileRows rows (Eq. 2 verbatim);
@@ -400,6 +518,7 @@ isp_status_t resolve_and_launch(Desc &d, int fam, int w, int h, int mw, int mh, 
     if (!direct && !d.g.vec_in && (chosen == ISP_BLOCK || chosen == ISP_WARP)) chosen = ISP_NAIVE;
     Plan p = plan_for(chosen);
     isp_plan_info info{};
+    const bool isp_degenerate = p.degenerate;
     if (p.degenerate) chosen = ISP_NAIVE;  // A3: Listing 3 cannot express a block needing opposite checks
     if (v == ISP_AUTO && !p.degenerate) {
         isp_model_params mp;
@@ -408,7 +527,8 @@ isp_status_t resolve_and_launch(Desc &d, int fam, int w, int h, int mw, int mh, 
         info.o_isp = chosen == ISP_TMA ? occupancy_of(nb_tma, tma_threads)
                                        : (nb_stream > 0 ? occupancy_of(nb_stream, threads) : 1.0);
         n_block(p, info.n_block);
-        model(p, w, h, mw, mh, mp, info);
+        if (chosen == ISP_TMA) mp.form = 2;   // staged kernels: checks per staged element (A21)
+        model(p, w, rr ? rr->nrows : h, mw, mh, mp, info);
         // Eq. (10) picks ISP iff G > 1.  B200 calibration (reading A29): the
         // u8 streaming fat kernels lose to naive below G ~ 2.4 (instruction-cache footprint
         // of nine bodies, which the model does not count), so AUTO requires G > 2.4 there.
@@ -429,17 +549,27 @@ isp_status_t resolve_and_launch(Desc &d, int fam, int w, int h, int mw, int mh, 
     d.g.sw = sg.sw;
     d.g.stages = sg.stages;
     d.g.rs = sg.rs;
+    d.g.tail = sg.tail;
     d.grid = dim3(p.nx, p.ny, 1);
     d.block = dim3(chosen == ISP_TMA ? tma_threads : threads, 1, 1);
     d.smem = chosen == ISP_TMA ? tma_smem : 0;
+    if (chosen == ISP_TMA && use_p) {
+        const long long nunits = (long long)p.nx * p.ny;
+        d.g.nux = p.nx;
+        d.g.nwc = nwc;
+        d.g.px = px;
+        d.g.nunits = (int)nunits;
+        d.g.sched = sched;
+        d.grid = dim3((unsigned)std::min<long long>(nunits, (long long)num_sms() * nb_tma), 1, 1);
+    }
     info.bh_l = p.bh_l; info.bh_r = p.bh_r; info.bh_t = p.bh_t; info.bh_b = p.bh_b;
     info.nx = p.nx; info.ny = p.ny; info.w_l = p.w_l; info.w_r = p.w_r;
-    info.degenerate = p.degenerate;
+    info.degenerate = p.degenerate || isp_degenerate;   // the ISP plan's, when it forced NAIVE
     info.tile_w = p.tile_w; info.tile_h = p.ty > 0 ? p.ty : (int)ceil_div(d.g.y_end - d.g.oy0, p.ny);
     info.warp_w = p.warp_w;
     n_block(p, info.n_block);
     info.choice = chosen;
-    d.disp = chosen == ISP_TMA ? DISP_TMA : chosen == ISP_WARP ? DISP_WARP : chosen == ISP_BLOCK ? DISP_BLOCK
+    d.disp = chosen == ISP_TMA ? tma_disp : chosen == ISP_WARP ? DISP_WARP : chosen == ISP_BLOCK ? DISP_BLOCK
                                                                                                : naive_disp;
     d.g.warp_level = chosen == ISP_WARP;
     d.g.mode = d.mode;

@@ -6,7 +6,7 @@
 
 #include "isp_direct.cuh"
 #include "isp_ops.cuh"
-#include "isp_staged.cuh"
+#include "isp_pstaged.cuh"
 #include "kernels.h"
 
 namespace ispk {
@@ -29,7 +29,10 @@ const void *kernel_for_disp(int disp)
     } else {
         switch (disp) {
         case DISP_TMA:
-            if constexpr (!Op::ROW_DIRECT) return (const void *)k_staged<Op>;  // one kernel, all modes
+            if constexpr (!Op::ROW_DIRECT) return (const void *)k_pstaged<Op>;  // one kernel, all modes
+            else return nullptr;
+        case DISP_TMA_STATIC:
+            if constexpr (!Op::ROW_DIRECT) return (const void *)k_staged<Op>;
             else return nullptr;
         case DISP_BLOCK: return (const void *)k_stencil<Op, MODE, DISP_BLOCK>;
         case DISP_WARP: return (const void *)k_stencil<Op, MODE, DISP_BLOCK>;

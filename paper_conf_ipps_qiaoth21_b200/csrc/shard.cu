@@ -34,9 +34,27 @@ isp_status_t nccl_status(ncclResult_t r, const char *what)
     return ispi_fail(ISP_ENCCL, "%s: %s", what, ncclGetErrorString(r));
 }
 
-template <class T> ncclDataType_t nccl_type();
-template <> ncclDataType_t nccl_type<float>() { return ncclFloat32; }
-template <> ncclDataType_t nccl_type<uint8_t>() { return ncclUint8; }
+
+// The halo exchange of one rank: the schedule's NCCL send/recv calls (bytes of `esz`-byte
+// elements, rows of `pitch` elements) in one group on `comm`.
+isp_status_t post_exchange(isp_shard_ctx *ctx, const isp_shard_sched &sc, void *strip, size_t esz, int pitch,
+                           cudaStream_t comm)
+{
+    isp_status_t s;
+    if ((s = nccl_status(ncclGroupStart(), "ncclGroupStart")) != ISP_OK) return s;
+    for (int k = 0; k < sc.n_ops; ++k) {
+        const isp_shard_op &op = sc.ops[k];
+        char *buf = (char *)strip + (size_t)op.row * pitch * esz;
+        const size_t cnt = (size_t)op.nrows * pitch * esz;
+        ncclResult_t r = op.kind == 0 ? ncclSend(buf, cnt, ncclUint8, op.peer, ctx->comm, comm)
+                                      : ncclRecv(buf, cnt, ncclUint8, op.peer, ctx->comm, comm);
+        if (r != ncclSuccess) {
+            ncclGroupEnd();
+            return nccl_status(r, op.kind == 0 ? "ncclSend" : "ncclRecv");
+        }
+    }
+    return nccl_status(ncclGroupEnd(), "ncclGroupEnd");
+}
 
 // ctx == nullptr: local mode (no exchange; the caller filled the halo rows).
 template <class T, class F>
@@ -50,24 +68,11 @@ isp_status_t shard_run(isp_shard_ctx *ctx, int rank, int nranks, T *strip, int w
     if (s != ISP_OK) return s;
     if (!ctx) sc.n_ops = 0;
     if (ctx && cudaSetDevice(ctx->device) != cudaSuccess) return ispi_fail(ISP_ECUDA, "cudaSetDevice");
-    const size_t row_elems = (size_t)pitch;
     if (sc.n_ops > 0) {
         if (cudaEventRecord(ctx->ev_ready, stream) != cudaSuccess ||
             cudaStreamWaitEvent(comm, ctx->ev_ready, 0) != cudaSuccess)
             return ispi_fail(ISP_ECUDA, "event record/wait");
-        if ((s = nccl_status(ncclGroupStart(), "ncclGroupStart")) != ISP_OK) return s;
-        for (int k = 0; k < sc.n_ops; ++k) {
-            const isp_shard_op &op = sc.ops[k];
-            T *buf = strip + (size_t)op.row * row_elems;
-            const size_t cnt = (size_t)op.nrows * row_elems;
-            ncclResult_t r = op.kind == 0 ? ncclSend(buf, cnt, nccl_type<T>(), op.peer, ctx->comm, comm)
-                                          : ncclRecv(buf, cnt, nccl_type<T>(), op.peer, ctx->comm, comm);
-            if (r != ncclSuccess) {
-                ncclGroupEnd();
-                return nccl_status(r, op.kind == 0 ? "ncclSend" : "ncclRecv");
-            }
-        }
-        if ((s = nccl_status(ncclGroupEnd(), "ncclGroupEnd")) != ISP_OK) return s;
+        if ((s = post_exchange(ctx, sc, strip, sizeof(T), pitch, comm)) != ISP_OK) return s;
         if (cudaEventRecord(ctx->ev_halo, comm) != cudaSuccess) return ispi_fail(ISP_ECUDA, "event record");
     }
     // global-row addressing: buffer row k holds global row y0 - halo + k
@@ -209,6 +214,17 @@ isp_status_t isp_shard_filter_local_u8(uint8_t *strip, int w, int H, int pitch, 
     };
     return shard_run<uint8_t>(nullptr, rank, nranks, strip, w, H, pitch, halo, mh / 2, border_mode, out, out_pitch,
                               (cudaStream_t)stream, (cudaStream_t)stream, f);
+}
+
+isp_status_t isp_shard_exchange(isp_shard_ctx *ctx, void *strip, int elem_size, int H, int pitch, int halo, int hy,
+                                int border_mode, isp_stream_t comm_stream)
+{
+    if (!ctx || !strip || elem_size < 1 || pitch < 1) return ispi_fail(ISP_EINVAL, "isp_shard_exchange args");
+    isp_shard_sched sc;
+    isp_status_t s = isp_shard_schedule(H, ctx->rank, ctx->nranks, halo, hy, border_mode, &sc);
+    if (s != ISP_OK) return s;
+    if (cudaSetDevice(ctx->device) != cudaSuccess) return ispi_fail(ISP_ECUDA, "cudaSetDevice");
+    return sc.n_ops > 0 ? post_exchange(ctx, sc, strip, (size_t)elem_size, pitch, (cudaStream_t)comm_stream) : ISP_OK;
 }
 
 isp_status_t isp_shard_destroy(isp_shard_ctx *ctx)

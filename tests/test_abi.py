@@ -142,3 +142,43 @@ def test_pipeline_cfg3_validation():
     assert call(hc=1021) == 1 and call(hc=-1021) == 1       # outside the Sobel range
     assert call(mag=FAKE_IN + 100) == 3                     # EALIAS
     assert call(dx=FAKE_IN + 64 * 63) == 3                  # int16 output overlapping the image tail
+
+
+def _balanced_y0s(h, ny, edge_w=64):
+    """Block-row starts of the library's balanced one-wave split (isp_core.cuh block_rows:
+    the first and last strip carry edge_w/256 of an interior strip's rows) -- the launch
+    geometry the model is evaluated on, restated here independently of the library."""
+    if ny <= 2:
+        return [(by * h) // ny for by in range(ny + 1)]
+    W = 2 * edge_w + 256 * (ny - 2)
+
+    def cum(k):
+        return 0 if k == 0 else W if k == ny else edge_w + 256 * (k - 1)
+    return [(cum(k) * h) // W for k in range(ny + 1)]
+
+
+@pytest.mark.parametrize("w,h,m", [(4096, 4096, 5), (2048, 1000, 7), (1000, 4096, 13), (4096, 512, 3)])
+@pytest.mark.parametrize("form", [0, 1, 2])
+def test_model_balanced_split_matches_oracle(w, h, m, form):
+    """Balanced one-wave plans (tile_h = 0): bounds from the real block-row starts and the
+    model counting each block's real rows (round-1 counted 0 pixels per block there)."""
+    mp = isp.ModelParams(4.0, 20.0, 2.0, 0.75, 0.5, form)
+    got = isp.isp_plan(w, h, m, m, tile_w=512, tile_h=0, warp_w=512, params=mp)
+    y0s = _balanced_y0s(h, got["ny"])
+    b = P.bounds_rows(w, h, m, m, 512, y0s)
+    assert (got["bh_t"], got["bh_b"], got["nx"], got["ny"]) == (b["BH_T"], b["BH_B"], b["NX"], b["NY"])
+    ref = P.model(w, h, m, m, 512, None, 4.0, 20.0, o_naive=0.75, o_isp=0.5, ipc_switch=2.0,
+                  form="TPS"[form], threads_per_block=32, y0s=y0s)
+    for k_got, k_ref in [("n_naive", "N_naive"), ("n_isp", "N_ISP"), ("r_reduced", "R_reduced"), ("g", "G")]:
+        assert got[k_got] == pytest.approx(ref[k_ref], rel=1e-12), k_got
+    assert got["n_isp"] > 0 and got["g"] < 100      # round 1: pix = 0 made G ~ 855
+
+
+def test_model_form_s_matches_oracle():
+    mp = isp.ModelParams(4.0, 20.0, 2.0, 0.75, 0.5, 2)
+    for (w, m, tw, th) in [(512, 13, 32, 4), (2048, 13, 128, 1), (4096, 5, 512, 32), (4096, 7, 1024, 16)]:
+        got = isp.isp_plan(w, w, m, m, tile_w=tw, tile_h=th, warp_w=tw, params=mp)
+        ref = P.model(w, w, m, m, tw, th, 4.0, 20.0, o_naive=0.75, o_isp=0.5, ipc_switch=2.0, form="S",
+                      threads_per_block=32)
+        assert got["n_isp"] == pytest.approx(ref["N_ISP"], rel=1e-12)
+        assert got["g"] == pytest.approx(ref["G"], rel=1e-12)

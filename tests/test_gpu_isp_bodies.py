@@ -406,7 +406,7 @@ def test_sobel_magnitude_near_ties(isp):
     nb = len(targets)
     per_row = 680
     rows = -(-nb // per_row)
-    img = np.zeros((3 * rows + 6, 3 * per_row + 24), dtype=np.uint8)   # 2064 wide: 16-B aligned rows
+    img = np.zeros((3 * rows + 40, 3 * per_row + 24), dtype=np.uint8)   # 2064 wide: 16-B aligned rows
     centres = []
     for t, (X, Y, n) in enumerate(targets):
         by, bx = 3 + 3 * (t // per_row), 3 * (t % per_row)

@@ -7,6 +7,7 @@ tests/golden/ and executed literally, and closed-form limits of the model.
 import os
 import re
 
+import numpy as np
 import pytest
 
 from oracle import planner as P
@@ -191,3 +192,80 @@ def test_model_limits():
     rp = P.model(4096, 4096, m, n, 32, 4, c, k, ipc_switch=ipc, form="P")["R_reduced"]
     assert abs(rp - (4 * c + k) / (ipc * 8 + k)) / rp < 0.02
     assert P.model(64, 64, 3, 3, 64, 8, c, k)["choice"] == "naive"      # degenerate
+
+
+# ---------------------------------------------------------------- block rows of any height
+def _needed_rows_bruteforce(sx, sy, m, n, tx, y0, y1, bx):
+    """Which checks block (bx, rows [y0, y1)) needs: every launched thread x every tap."""
+    hx, hy = m // 2, n // 2
+    need = set()
+    for y in range(y0, y1):
+        for x in range(bx * tx, (bx + 1) * tx):
+            for j in range(n):
+                for i in range(m):
+                    xx, yy = x + i - hx, y + j - hy
+                    if xx < 0:
+                        need.add("L")
+                    if xx >= sx:
+                        need.add("R")
+                    if yy < 0:
+                        need.add("T")
+                    if yy >= sy:
+                        need.add("B")
+    return need
+
+
+def test_bounds_rows_bruteforce():
+    """bounds_rows (Eq. 2 for block rows of any height, e.g. the balanced one-wave split)
+    is conservative and tight against per-thread enumeration: a block row < BH_T needs
+    the T check and none >= BH_T does; likewise B."""
+    rng = np.random.default_rng(3)
+    for _ in range(60):
+        sy = int(rng.integers(4, 40))
+        n = int(rng.choice([1, 3, 5, 7]))
+        cuts = sorted(set(int(c) for c in rng.integers(1, sy, int(rng.integers(1, 6)))))
+        y0s = [0] + cuts + [sy]
+        sx, m, tx = 8, 3, 8
+        b = P.bounds_rows(sx, sy, m, n, tx, y0s)
+        for by in range(len(y0s) - 1):
+            need = _needed_rows_bruteforce(sx, sy, m, n, tx, y0s[by], y0s[by + 1], 0)
+            assert ("T" in need) == (by < b["BH_T"]), (y0s, n, by, b)
+            assert ("B" in need) == (by >= b["BH_B"]), (y0s, n, by, b)
+
+
+@pytest.mark.parametrize("sx,sy,m,tx,ty", [(512, 512, 13, 32, 4), (300, 77, 5, 64, 8), (4096, 4096, 5, 512, 32)])
+def test_bounds_rows_uniform_equals_eq2(sx, sy, m, tx, ty):
+    NY = -(-sy // ty)
+    y0s = [min(sy, by * ty) for by in range(NY + 1)]
+    b, bu = P.bounds_rows(sx, sy, m, m, tx, y0s), P.bounds(sx, sy, m, m, tx, ty)
+    # identical except where the uniform model's last partial tile ends past the image
+    assert {k: b[k] for k in ("BH_L", "BH_R", "BH_T", "NX", "NY")} == {k: bu[k] for k in ("BH_L", "BH_R", "BH_T", "NX", "NY")}
+    assert b["BH_B"] == bu["BH_B"] or (sy % ty and b["BH_B"] >= bu["BH_B"])
+
+
+def test_model_rows_reduces_to_printed_form():
+    """y0s of uniform full tiles give exactly the printed Eq. (5) sum."""
+    for (s, m, tx, ty) in [(512, 13, 32, 4), (1024, 5, 128, 8)]:
+        y0s = [by * ty for by in range(s // ty + 1)]
+        for form in ("T", "P", "S"):
+            a = P.model(s, s, m, m, tx, ty, 4.0, 20.0, form=form, threads_per_block=32)
+            b = P.model(s, s, m, m, tx, ty, 4.0, 20.0, form=form, threads_per_block=32, y0s=y0s)
+            assert a["N_ISP"] == pytest.approx(b["N_ISP"], rel=1e-12)
+
+
+def test_model_form_s_closed_form():
+    """Form S (reading A21) on a 3x3-block image: 8 border blocks (4 corners x 2 checks,
+    4 edges x 1) pay n_check per staged element (tx+2hx)(ty+2hy); Body pays none;
+    with n_check = 0 it equals form T with n_check = 0."""
+    sx = sy = 48
+    m = n = 5
+    tx = ty = 16
+    c, k, ipc, thr = 3.0, 7.0, 2.0, 64
+    got = P.model(sx, sy, m, n, tx, ty, c, k, ipc_switch=ipc, form="S", threads_per_block=thr)
+    sw = P.n_switch_table()
+    E = (tx + 4) * (ty + 4)
+    want = sum(sw[r] * ipc * thr for r in P.REGIONS) + (4 * 2 + 4 * 1) * c * E + 9 * k * m * n * tx * ty
+    assert got["N_ISP"] == pytest.approx(want, rel=1e-12)
+    a = P.model(sx, sy, m, n, tx, ty, 0.0, k, form="S", threads_per_block=thr)
+    b = P.model(sx, sy, m, n, tx, ty, 0.0, k, form="T", threads_per_block=thr)
+    assert a["N_ISP"] == pytest.approx(b["N_ISP"], rel=1e-12)
