@@ -186,6 +186,19 @@ typedef struct {
  * 6 bilateral, 7 atrous.  tile_w/tile_h <= 0 selects the library's launch tile. */
 isp_status_t isp_plan(int w, int h, int mw, int mh, int tile_w, int tile_h, int warp_w, int border_mode,
                       int filter_id, const isp_model_params *params, isp_plan_info *out);
+/* Sparse masks (the paper's future work P:L394; reading A31).  reach =
+ * {left, right, top, bottom}: how far the NON-ZERO taps of an odd mw x mh mask reach
+ * beyond its centre anchor (clamped at 0).  isp_filter_ex / isp_filter_u8 crop masks with
+ * all-zero edge rows / columns to this footprint (zero taps add exactly 0 on finite
+ * images, so results are unchanged) and take the ISP bounds from it.  dtype: ISP_F32
+ * (float mask) or ISP_I32 (int32 mask).  Pure host. */
+isp_status_t isp_mask_reach(const void *mask, int dtype, int mw, int mh, int reach[4]);
+/* Eq. (2) with per-side reaches (reading A31): BH_L = ceil(L/tx), BH_R = floor((w-R)/tx),
+ * BH_T = ceil(T/ty), BH_B = floor((h-B)/ty), warp bounds likewise, Eq. (8) block counts.
+ * tile_w = tx (pixels), tile_h = ty (rows), warp_w = warp width in pixels (<= 0: tx).
+ * Pure host; model fields are not filled (choice = ISP_BLOCK, or ISP_NAIVE if degenerate). */
+isp_status_t isp_plan_reach(int w, int h, const int reach[4], int tile_w, int tile_h, int warp_w,
+                            isp_plan_info *out);
 /* Default model constants for a filter/mode (calibration). */
 isp_status_t isp_model_defaults(int filter_id, int border_mode, int mw, int mh, isp_model_params *out);
 

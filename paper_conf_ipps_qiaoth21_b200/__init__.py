@@ -24,7 +24,7 @@ __all__ = [
     "lib", "IspError", "PlanInfo", "ModelParams",
     "isp_filter", "isp_filter_naive", "isp_filter_ex", "isp_filter_sep_f32", "isp_filter_u8",
     "isp_sobel_u8", "isp_laplace5_u8", "isp_harris_u8", "isp_pipeline_cfg3_u8", "isp_bilateral_f32", "isp_atrous_f32",
-    "isp_night_f32", "isp_plan", "isp_model_defaults", "isp_last_plan", "isp_recent_plans", "isp_clear_plans",
+    "isp_night_f32", "isp_plan", "isp_model_defaults", "isp_mask_reach", "isp_plan_reach", "isp_last_plan", "isp_recent_plans", "isp_clear_plans",
     "isp_set_launch_override",
     "isp_shard_unique_id", "isp_shard_init", "isp_shard_rows", "isp_shard_schedule",
     "isp_shard_filter_f32", "isp_shard_filter_u8", "isp_shard_filter_local_f32", "isp_shard_filter_local_u8",
@@ -116,6 +116,8 @@ _SIGS = {
     "isp_shard_filter_local_u8": [_P, _I, _I, _I, _I, _I, _I, _P, _I, _I, ctypes.c_int32, _I, _I, _P, _I, _I, _P],
     "isp_recent_plans": [_P, _I],
     "isp_shard_exchange": [_P, _P, _I, _I, _I, _I, _I, _I, _P],
+    "isp_mask_reach": [_P, _I, _I, _I, _P],
+    "isp_plan_reach": [_I, _I, _P, _I, _I, _I, _P],
 }
 
 _lib = None
@@ -363,6 +365,24 @@ def isp_plan(w, h, mw, mh, tile_w=0, tile_h=0, warp_w=0, border_mode=CLAMP, filt
     pp = ctypes.byref(params) if params is not None else None
     _check(lib().isp_plan(int(w), int(h), int(mw), int(mh), int(tile_w), int(tile_h), int(warp_w),
                           _mode(border_mode), int(filter_id), pp, ctypes.byref(info)))
+    return info.as_dict()
+
+
+def isp_mask_reach(mask):
+    """(left, right, top, bottom) reach of the mask's non-zero taps (reading A31)."""
+    import numpy as np
+    m = np.asarray(mask)
+    is_int = np.issubdtype(m.dtype, np.integer)
+    a, ap = _host(m, ctypes.c_int32 if is_int else ctypes.c_float)
+    r = (ctypes.c_int * 4)()
+    _check(lib().isp_mask_reach(ap, 2 if is_int else 3, a.shape[1], a.shape[0], r))
+    return tuple(r)
+
+
+def isp_plan_reach(w, h, reach, tile_w, tile_h, warp_w=0):
+    r = (ctypes.c_int * 4)(*[int(x) for x in reach])
+    info = PlanInfo()
+    _check(lib().isp_plan_reach(int(w), int(h), r, int(tile_w), int(tile_h), int(warp_w), ctypes.byref(info)))
     return info.as_dict()
 
 

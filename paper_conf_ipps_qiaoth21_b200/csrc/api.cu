@@ -115,9 +115,13 @@ constexpr int kMinRowsPerBlock = 8;
 constexpr int kStreamTileRows = 16;
 
 // blocks_per_sm: resident blocks of the kernel that will run (occupancy API); 0 = 8.
+// hx, hy: reach of the window to the left / top of the anchor; hxr, hyb (default hx, hy):
+// to the right / bottom -- the non-zero footprint of a sparse mask (reading A31).
 Plan make_plan(int w, int h, int hx, int hy, int px, int tile_w_req, int tile_h_req, int warp_w_req,
-               const RowRange *rr = nullptr, int blocks_per_sm = 0)
+               const RowRange *rr = nullptr, int blocks_per_sm = 0, int hxr = -1, int hyb = -1)
 {
+    if (hxr < 0) hxr = hx;
+    if (hyb < 0) hyb = hy;
     const RowRange whole{0, h, h, 1, 1};
     if (!rr) rr = &whole;
     Plan p{};
@@ -150,13 +154,13 @@ Plan make_plan(int w, int h, int hx, int hy, int px, int tile_w_req, int tile_h_
         p.ny = (int)nby;
     }
     p.bh_l = (int)ceil_div(hx, p.tile_w);
-    p.bh_r = (int)floor_div(w - hx, p.tile_w);
+    p.bh_r = (int)floor_div(w - hxr, p.tile_w);
     p.w_l = (int)ceil_div(hx, warp_w);
-    p.w_r = (int)floor_div(w - hx, warp_w);
+    p.w_r = (int)floor_div(w - hxr, warp_w);
     // Eq. (2) in y, relative to the launch's first row oy0; only real image edges count.
     if (p.ty > 0) {
         p.bh_t = rr->t_real ? (int)std::max<long long>(0, ceil_div(hy - rr->oy0, p.ty)) : 0;
-        const long long safe_end = rr->b_real ? std::min<long long>(rr->oy0 + nr, (long long)h - hy)
+        const long long safe_end = rr->b_real ? std::min<long long>(rr->oy0 + nr, (long long)h - hyb)
                                               : rr->oy0 + nr;
         p.bh_b = (int)floor_div(safe_end - rr->oy0, p.ty);
     } else {
@@ -176,7 +180,7 @@ Plan make_plan(int w, int h, int hx, int hy, int px, int tile_w_req, int tile_h_
             while (bt < p.ny && y0_of(bt) - hy < 0) ++bt;
         int bb = p.ny;
         if (rr->b_real)
-            while (bb > 0 && y0_of(bb) + hy > h) --bb;   // y0_of(bb) = end of block bb-1
+            while (bb > 0 && y0_of(bb) + hyb > h) --bb;   // y0_of(bb) = end of block bb-1
         p.bh_t = bt;
         p.bh_b = bb;
         if (bt <= bb) {
@@ -383,8 +387,8 @@ StagedGeom staged_geom(int w, int hx, int hy, int px, int esz, int nin, int nwc 
     const long long slot_bytes = row_bytes * sg.rs;
     sg.stages = (int)std::min<long long>(32, std::max<long long>(4, ceil_div(8 * 1024, slot_bytes)));
     if (const char *e = getenv("ISP_STAGES")) sg.stages = std::max(2, std::min(32, atoi(e)));
-    sg.tail = env_int("ISP_TAIL", 1, 0, 1);
-    sg.smem = 640 + (size_t)sg.stages * slot_bytes + (sg.tail ? (size_t)2 * hy * row_bytes : 0);
+    sg.tail = 0;   // tail prefetch: rejected
+    sg.smem = 512 + (size_t)sg.stages * slot_bytes;
     return sg;
 }
 
@@ -451,9 +455,13 @@ isp_status_t resolve_and_launch(Desc &d, int fam, int w, int h, int mw, int mh, 
         d.g.t_real = rr->t_real;
         d.g.b_real = rr->b_real;
     }
-    const Plan p0 = make_plan(w, h, hx, hy, px, 0, 0, 0, rr, 0);
+    // reaches of the window (left, right, top, bottom): the non-zero footprint of a
+    // cropped sparse mask (reading A31), else hx / hy on both sides
+    const int rl = d.has_reach ? d.reach[0] : hx, rrx = d.has_reach ? d.reach[1] : hx;
+    const int rt = d.has_reach ? d.reach[2] : hy, rb = d.has_reach ? d.reach[3] : hy;
+    const Plan p0 = make_plan(w, h, rl, rt, px, 0, 0, 0, rr, 0, rrx, rb);
     const int threads = 32 * p0.wx;
-    const bool fits = hx <= w && hy <= h;  // one reflection suffices (naive Mirror)
+    const bool fits = std::max(rl, rrx) <= w && std::max(rt, rb) <= h;  // one reflection suffices (naive Mirror)
     const int naive_disp = fits ? DISP_NAIVE : DISP_NAIVE_GEN;
     auto fn_of = [&](int disp) {
         Desc q = d;
@@ -473,7 +481,7 @@ isp_status_t resolve_and_launch(Desc &d, int fam, int w, int h, int mw, int mh, 
     if (direct) tma_ok = true;
     tma_ok = tma_ok && fn_of(tma_disp) != nullptr && g_override_wx == 0;
     const int tma_threads = direct ? TILE_THREADS : 32 * (nwc + 1);
-    const size_t tma_smem = direct ? (size_t)(TILE_PX * 32 + 2 * hx) * (TILE_H + 2 * hy) * esz : sg.smem;
+    const size_t tma_smem = direct ? (size_t)(TILE_PX * 32 + d.mw - 1) * (TILE_H + d.mh - 1) * esz : sg.smem;
     const int nb_naive = blocks_per_sm(fn_of(naive_disp), threads);
     const int nb_stream = blocks_per_sm(fn_of(p0.wx > 1 ? DISP_WARP : DISP_BLOCK), threads);
     int nb_tma = tma_ok ? blocks_per_sm(fn_of(tma_disp), tma_threads, tma_smem) : 0;
@@ -489,7 +497,7 @@ isp_status_t resolve_and_launch(Desc &d, int fam, int w, int h, int mw, int mh, 
     if (v == ISP_AUTO) chosen = (tma_ok && esz == 4) ? ISP_TMA : (p0.wx > 1 ? ISP_WARP : ISP_BLOCK);
     auto plan_for = [&](isp_variant_t c) {
         if (c == ISP_TMA && direct)  // tiles of TILE_PX*32 x TILE_H, Eq. (2) verbatim
-            return make_plan(w, h, hx, hy, px, TILE_PX * 32, TILE_H, TILE_PX * 32, rr, nb_tma);
+            return make_plan(w, h, rl, rt, px, TILE_PX * 32, TILE_H, TILE_PX * 32, rr, nb_tma, rrx, rb);
         if (c == ISP_TMA) {
             // persistent: uniform tiles of nwc*32*px x CH (Eq. 2 verbatim in y);
             // static: the balanced one-wave row split
@@ -510,8 +518,8 @@ isp_status_t resolve_and_launch(Desc &d, int fam, int w, int h, int mw, int mh, 
         int ty = kStreamTileRows;
         const int nrw = rr ? rr->nrows : h;
         while (ty > 1 && (long long)p0.nx * ceil_div(nrw, ty) < num_sms()) ty /= 2;
-        return make_plan(w, h, hx, hy, px, 0, g_override_ty > 0 ? 0 : ty, 0, rr,
-                         c == ISP_NAIVE ? nb_naive : nb_stream);
+        return make_plan(w, h, rl, rt, px, 0, g_override_ty > 0 ? 0 : ty, 0, rr,
+                         c == ISP_NAIVE ? nb_naive : nb_stream, rrx, rb);
     };
     // the streaming ISP bodies assume vector-aligned rows (isp_core.cuh load_row):
     // misaligned images run the naive kernel (identical results)
@@ -732,6 +740,55 @@ isp_status_t isp_set_launch_override(int warps_x, int tile_h)
 
 }  // extern "C"
 
+// ---------------------------------------------------------------------------------
+// Sparse masks (the paper's future work), reading A31: a mask
+// with all-zero edge rows / columns is cropped to its non-zero footprint.  Zero taps add
+// exactly 0 (finite images), so the cropped window computes the same bits; the ISP
+// bounds (Eq. 2) then follow the footprint's reach on each side instead of the bounding
+// window.  A footprint that is still a centred odd 3/5/7 square runs the compiled
+// kernels; any other footprint runs the direct family with its anchor (ax, ay).
+// ---------------------------------------------------------------------------------
+struct Crop {
+    bool cropped = false;
+    int mw, mh, ax, ay;     // cropped window and anchor
+    int reach[4];           // L, R, T, B (clamped at 0: partial tiles stay in R / B, A10)
+    bool centred() const { return ax == mw - 1 - ax && ay == mh - 1 - ay; }
+};
+
+template <class M>
+Crop crop_mask(const M *mask, int mw, int mh, std::vector<M> &out)
+{
+    Crop c;
+    c.mw = mw;
+    c.mh = mh;
+    c.ax = mw / 2;
+    c.ay = mh / 2;
+    int i0 = mw, i1 = -1, j0 = mh, j1 = -1;
+    for (int j = 0; j < mh; ++j)
+        for (int i = 0; i < mw; ++i)
+            if (mask[j * mw + i] != M(0)) {
+                i0 = std::min(i0, i); i1 = std::max(i1, i);
+                j0 = std::min(j0, j); j1 = std::max(j1, j);
+            }
+    if (i1 < 0) { i0 = i1 = mw / 2; j0 = j1 = mh / 2; }     // all zero: the centre tap (weight 0)
+    c.reach[0] = std::max(0, mw / 2 - i0);
+    c.reach[1] = std::max(0, i1 - mw / 2);
+    c.reach[2] = std::max(0, mh / 2 - j0);
+    c.reach[3] = std::max(0, j1 - mh / 2);
+    if (i0 == 0 && i1 == mw - 1 && j0 == 0 && j1 == mh - 1) return c;
+    c.cropped = true;
+    c.mw = i1 - i0 + 1;
+    c.mh = j1 - j0 + 1;
+    c.ax = mw / 2 - i0;
+    c.ay = mh / 2 - j0;
+    out.resize((size_t)c.mw * c.mh);
+    for (int j = 0; j < c.mh; ++j)
+        for (int i = 0; i < c.mw; ++i) out[(size_t)j * c.mw + i] = mask[(j + j0) * mw + i + i0];
+    return c;
+}
+
+bool compiled_window(int mw, int mh) { return mw == mh && (mw == 3 || mw == 5 || mw == 7); }
+
 // Internal row-range entry points (multi-GPU strips, shard.cu).  `img` is addressed
 // with global rows; `out` points at the output row rr->oy0.
 isp_status_t ispi_filter_f32(const float *img, int w, int h, int pitch, const float *mask, int mw, int mh,
@@ -751,8 +808,26 @@ isp_status_t ispi_filter_f32(const float *img, int w, int h, int pitch, const fl
     d.mh = mh;
     d.g.vec_in = aligned(img, (long long)pitch * 4, 16);
     d.g.vec_out = aligned(out, (long long)out_pitch * 4, 16);
+    std::vector<float> cm;
+    const Crop cr = crop_mask(mask, mw, mh, cm);
+    if (cr.cropped) {   // sparse mask: its non-zero footprint (reading A31)
+        if (cr.centred() && compiled_window(cr.mw, cr.mh))
+            return ispi_filter_f32(img, w, h, pitch, cm.data(), cr.mw, cr.mh, border_mode, const_val, out, out_pitch,
+                                   variant, stream, rr);
+        d.mw = cr.mw;
+        d.mh = cr.mh;
+        d.ax = cr.ax;
+        d.ay = cr.ay;
+        std::memcpy(d.reach, cr.reach, sizeof(d.reach));
+        d.has_reach = 1;
+        d.maskf = cm.data();
+        return resolve_and_launch(d, F_CONV_F32, w, h, cr.mw, cr.mh, cr.reach[0], cr.reach[2], true, variant,
+                                  kfn_dconv_f32, run_dconv_f32, "isp_filter(sparse mask)", rr);
+    }
+    d.ax = mw / 2;
+    d.ay = mh / 2;
     std::vector<float> row, col;
-    if (mw == mh && (mw == 3 || mw == 5 || mw == 7)) {
+    if (compiled_window(mw, mh)) {
         if (separable_f32(mask, mw, mh, row, col)) {
             d.rowf = row.data();
             d.colf = col.data();
@@ -790,6 +865,26 @@ isp_status_t ispi_filter_u8(const uint8_t *img, int w, int h, int pitch, const i
     d.mw = mw;
     d.mh = mh;
     d.rnd = make_round(divisor);
+    std::vector<int32_t> cm;
+    const Crop cr = crop_mask(mask, mw, mh, cm);
+    if (cr.cropped) {   // sparse mask: its non-zero footprint (reading A31)
+        if (cr.centred() && compiled_window(cr.mw, cr.mh))
+            return ispi_filter_u8(img, w, h, pitch, cm.data(), cr.mw, cr.mh, divisor, border_mode, const_val, out,
+                                  out_pitch, variant, stream, rr);
+        d.mw = cr.mw;
+        d.mh = cr.mh;
+        d.ax = cr.ax;
+        d.ay = cr.ay;
+        std::memcpy(d.reach, cr.reach, sizeof(d.reach));
+        d.has_reach = 1;
+        d.maski = cm.data();
+        d.g.vec_in = aligned(img, pitch, 4);
+        d.g.vec_out = aligned(out, out_pitch, 4);
+        return resolve_and_launch(d, F_U8, w, h, cr.mw, cr.mh, cr.reach[0], cr.reach[2], true, variant,
+                                  kfn_dconv_u8, run_dconv_u8, "isp_filter_u8(sparse mask)", rr);
+    }
+    d.ax = mw / 2;
+    d.ay = mh / 2;
     std::vector<int> row, col;
     if (mw == mh && (mw == 3 || mw == 5 || mw == 7)) {
         d.g.vec_in = aligned(img, pitch, 8);
@@ -861,6 +956,8 @@ isp_status_t isp_filter_sep_f32(const float *img, int w, int h, int pitch, const
     for (int j = 0; j < mh; ++j)
         for (int i = 0; i < mw; ++i) m2[j * mw + i] = col[j] * row[i];
     d.maskf = m2.data();
+    d.ax = mw / 2;
+    d.ay = mh / 2;
     return resolve_and_launch(d, F_SEP_F32, w, h, mw, mh, mw / 2, mh / 2, true, variant, kfn_dconv_f32,
                               run_dconv_f32, "isp_filter_sep_f32(direct)");
 }
@@ -973,6 +1070,7 @@ isp_status_t isp_bilateral_f32(const float *img, int w, int h, int pitch, int wi
             ls[j * win + i] = (float)(-r2 / (2.0 * (double)sigma_d * sigma_d) * LOG2E);
         }
     d.ls = ls.data();
+    d.ax = d.ay = hw;
     d.g.vec_in = 0;
     d.g.vec_out = aligned(out, (long long)out_pitch * 4, 16);
     return resolve_and_launch(d, F_BILATERAL, w, h, win, win, hw, hw, true, variant, kfn_bilateral, run_bilateral,
@@ -1013,6 +1111,42 @@ isp_status_t isp_night_f32(const float *img, int w, int h, int pitch, int border
     if ((s = isp_atrous_f32(tmp0, w, h, out_pitch, 2, border_mode, const_val, 0, tmp1, out_pitch, variant, stream))) return s;
     if ((s = isp_atrous_f32(tmp1, w, h, out_pitch, 4, border_mode, const_val, 0, tmp0, out_pitch, variant, stream))) return s;
     return isp_atrous_f32(tmp0, w, h, out_pitch, 8, border_mode, const_val, 1, out, out_pitch, variant, stream);
+}
+
+isp_status_t isp_mask_reach(const void *mask, int dtype, int mw, int mh, int reach[4])
+{
+    if (!mask || !reach || mw < 1 || mh < 1 || mw > 31 || mh > 31 || (mw % 2) == 0 || (mh % 2) == 0)
+        return fail(ISP_EINVAL, "isp_mask_reach args");
+    Crop c;
+    if (dtype == ISP_F32) {
+        std::vector<float> t;
+        c = crop_mask((const float *)mask, mw, mh, t);
+    } else if (dtype == ISP_I32) {
+        std::vector<int32_t> t;
+        c = crop_mask((const int32_t *)mask, mw, mh, t);
+    } else {
+        return fail(ISP_EINVAL, "dtype %d (ISP_F32 or ISP_I32)", dtype);
+    }
+    std::memcpy(reach, c.reach, sizeof(c.reach));
+    return ISP_OK;
+}
+
+isp_status_t isp_plan_reach(int w, int h, const int reach[4], int tile_w, int tile_h, int warp_w, isp_plan_info *out)
+{
+    if (!reach || !out || w < 1 || h < 1 || tile_w < 1 || tile_h < 1) return fail(ISP_EINVAL, "isp_plan_reach args");
+    for (int k = 0; k < 4; ++k)
+        if (reach[k] < 0 || reach[k] > 30) return fail(ISP_EINVAL, "reach[%d] = %d", k, reach[k]);
+    Plan p = make_plan(w, h, reach[0], reach[2], 1, tile_w, tile_h, warp_w > 0 ? warp_w : tile_w, nullptr, 0,
+                       reach[1], reach[3]);
+    isp_plan_info info{};
+    info.bh_l = p.bh_l; info.bh_r = p.bh_r; info.bh_t = p.bh_t; info.bh_b = p.bh_b;
+    info.nx = p.nx; info.ny = p.ny; info.w_l = p.w_l; info.w_r = p.w_r;
+    info.degenerate = p.degenerate;
+    info.tile_w = p.tile_w; info.tile_h = p.ty; info.warp_w = p.warp_w;
+    n_block(p, info.n_block);
+    info.choice = p.degenerate ? ISP_NAIVE : ISP_BLOCK;
+    *out = info;
+    return ISP_OK;
 }
 
 isp_status_t isp_model_defaults(int filter_id, int border_mode, int mw, int mh, isp_model_params *out)

@@ -32,7 +32,9 @@ __device__ __forceinline__ void direct_body(const typename Op::Params &p, int x0
     using T = typename Op::Tin;
     constexpr int PX = Op::PX;
     const Geom &g = p.g;
-    const int hx = p.mw / 2, hy = p.mh / 2;
+    // anchor (ax, ay): taps at offsets (i - ax, j - ay); the centre for dense windows,
+    // anywhere for cropped sparse masks (reading A31)
+    const int hx = p.ax, hy = p.ay;
     for (int o = 0; o < rows; ++o) {
         const int y = y0 + o;
         typename Op::A acc;
@@ -108,7 +110,7 @@ __device__ __forceinline__ void tile_fill(const typename Op::Params &p, typename
 {
     using T = typename Op::Tin;
     const Geom &g = p.g;
-    const int hx = p.mw / 2, hy = p.mh / 2;
+    const int hx = p.ax, hy = p.ay;
     for (int r = threadIdx.x / 32; r < SH; r += kTileWarps) {
         bool rowok;
         const int yy = map_row<MODE, CK>(Y0 - hy + r, g, rowok);
@@ -132,7 +134,7 @@ __device__ __forceinline__ void tile_body(const typename Op::Params &p, typename
     constexpr int PX = Op::PX, TW = 32 * PX;
     static_assert(PX == TILE_PX, "the planner sizes tiles with TILE_PX");
     const int X0 = blockIdx.x * TW, Y0 = p.g.oy0 + blockIdx.y * kTileH;
-    const int SW = TW + 2 * (p.mw / 2), SH = kTileH + 2 * (p.mh / 2);
+    const int SW = TW + p.mw - 1, SH = kTileH + p.mh - 1;
     tile_fill<Op, MODE, CK>(p, tile, X0, Y0, SW, SH);
     __syncthreads();
     const int lane = threadIdx.x & 31;
@@ -140,7 +142,7 @@ __device__ __forceinline__ void tile_body(const typename Op::Params &p, typename
         const int y = Y0 + o;
         if ((CK & CK_B) && y >= p.g.y_end) break;
         typename Op::A acc;
-        Op::init_tile(p, acc, tile + (o + p.mh / 2) * SW + p.mw / 2 + lane);
+        Op::init_tile(p, acc, tile + (o + p.ay) * SW + p.ax + lane);
         for (int j = 0; j < p.mh; ++j) {
             const T *srow = tile + (o + j) * SW + lane;
 #pragma unroll 2
@@ -196,6 +198,7 @@ struct DOpConvF32 {
         float cval;
         float *out;
         int mw, mh;
+        int ax, ay;   // anchor: tap (i, j) reads offset (i - ax, j - ay)
         float mask[MAXT];
     };
     struct A { float v[PX]; };
@@ -234,6 +237,7 @@ struct DOpConvU8 {
         uint8_t cval;
         uint8_t *out;
         int mw, mh;
+        int ax, ay;   // anchor: tap (i, j) reads offset (i - ax, j - ay)
         U8Round rnd;
         int mask[MAXT];
     };
@@ -279,6 +283,7 @@ struct DOpBilateral {
         float cval;
         float *out;
         int mw, mh;
+        int ax, ay;   // anchor: tap (i, j) reads offset (i - ax, j - ay)
         float kr;
         float ls[MAXT];  // log2 of the spatial weights s(dx, dy)
     };

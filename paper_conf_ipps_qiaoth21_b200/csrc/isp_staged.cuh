@@ -21,7 +21,7 @@ namespace ispk {
 constexpr int kStagedComputeWarps = 4;
 constexpr int kStagedThreads = 32 * (kStagedComputeWarps + 1);
 constexpr int kStagedMaxStages = 32;
-constexpr int kStagedBarrierBytes = 640;  // full[32] + empty[32] + tail mbarriers (+ pad to 128 B)
+constexpr int kStagedBarrierBytes = 512;  // full[32] + empty[32] mbarriers
 
 __device__ __forceinline__ uint32_t smem_u32(const void *p) { return (uint32_t)__cvta_generic_to_shared(p); }
 
@@ -180,114 +180,89 @@ __device__ __forceinline__ void staged_edge_fix(const Geom &g, int x0, typename 
     }
 }
 
-// One input row (CTA-relative input row f, global row y0 - HY + f) into shared memory at
-// rb: bulk copies of the in-bounds span (lane 0, completing on `bar` with its expect_tx),
-// this region's column fix-ups (all lanes; 4-byte types by cp.async, the caller arrives
-// for them), Constant rows outside the image filled with C.
+// Producer warp of a staged CTA (the only mode-dependent code: row maps, fix-ups).
 template <class Op, int MODE, int CK>
-__device__ __forceinline__ void staged_fill_row(const typename Op::Params &p, typename Op::Tin *rb, int yrow, int X0,
-                                                uint64_t *bar)
+__device__ __forceinline__ void staged_producer(const typename Op::Params &p, uint64_t *full, uint64_t *empty,
+                                                typename Op::Tin *buf, int y0, int nr, int X0)
 {
     using T = typename Op::Tin;
-    constexpr int PX = Op::PX, NIN = Op::NIN;
+    constexpr int HY = Op::HY, PX = Op::PX, NIN = Op::NIN;
     constexpr int TW = kStagedComputeWarps * 32 * PX;
     constexpr bool ASYNC_FIX = (CK & (CK_L | CK_R)) != 0 && sizeof(T) == 4 && MODE != CONSTANT;
     const Geom &g = p.g;
-    const int SW = g.sw, HXA = g.hxa;
+    const int S = g.stages, SW = g.sw, HXA = g.hxa, RS = g.rs;
     const int lane = threadIdx.x & 31;
     const int XS = X0 - HXA;
-    bool rowok;
-    const int yy = map_row<MODE, CK>(yrow, g, rowok);
-    int cs = XS, ce = X0 + TW + HXA;
-    if constexpr ((CK & CK_L) != 0) cs = max(cs, 0);
-    if constexpr ((CK & CK_R) != 0) ce = min(ce, g.w_al);
-    if (MODE == CONSTANT && !rowok) ce = cs;  // whole row = C
-    if (lane == 0 && ce > cs) {
-        mbar_expect_tx(bar, (uint32_t)(ce - cs) * (uint32_t)sizeof(T) * NIN);
-#pragma unroll
-        for (int c = 0; c < NIN; ++c)
-            bulk_g2s(rb + (size_t)c * SW + (cs - XS), p.in[c] + (ptrdiff_t)yy * g.in_pitch + cs,
-                     (uint32_t)(ce - cs) * (uint32_t)sizeof(T), bar);
-    }
-    if (CK != 0 && g.dbg != 4) {
-        // column fix-ups unless the compute warps rebuild the edge columns
-        const bool colfix = !((CK & (CK_L | CK_R)) && consumer_fix(g, PX));
-        // border fix-ups, this region's sides only (<= HXA columns per row): cp.async of
-        // the pattern's source column (4-byte types), else a synchronous copy; Constant:
-        // the constant
-#pragma unroll
-        for (int c = 0; c < NIN; ++c) {
-            T *dst = rb + (size_t)c * SW;
-            if (MODE == CONSTANT && !rowok) {
-                for (int x = lane; x < SW; x += 32) dst[x] = p.cval;
-                continue;
-            }
-            if (!colfix) continue;
-            const T *src = p.in[c] + (ptrdiff_t)yy * g.in_pitch;
-            auto fix = [&](int x) {
-                if constexpr (MODE == CONSTANT) {
-                    dst[x - XS] = (x >= 0 && x < g.w) ? __ldg(src + x) : p.cval;
-                } else {
-                    const int xs = fixup_source<Op, MODE, CK>(x, g);
-                    if (xs < 0) return;
-                    if constexpr (ASYNC_FIX) cp_async4(dst + (x - XS), src + xs);
-                    else dst[x - XS] = __ldg(src + xs);
-                }
-            };
-            if constexpr ((CK & CK_L) != 0)
-                for (int x = XS + lane; x < cs; x += 32) fix(x);
-            if constexpr ((CK & CK_R) != 0)
-                for (int x = ce + lane; x < X0 + TW + HXA; x += 32) fix(x);
-        }
-    }
-}
-
-// Arrivals that close one fill of `bar` (after staged_fill_row calls).
-template <class Op, int MODE, int CK>
-__device__ __forceinline__ void staged_fill_done(const typename Op::Params &p, uint64_t *bar)
-{
-    using T = typename Op::Tin;
-    constexpr bool ASYNC_FIX = (CK & (CK_L | CK_R)) != 0 && sizeof(T) == 4 && MODE != CONSTANT;
-    const Geom &g = p.g;
-    if constexpr (ASYNC_FIX) {
-        if (g.dbg != 4 && !consumer_fix(g, Op::PX)) cp_async_mbar_arrive_noinc(bar);
-    }
-    if constexpr (MODE == CONSTANT && (CK & (CK_T | CK_B)) != 0)
-        fence_proxy_async();  // generic row fills before later bulk (async-proxy) writes
-    __syncwarp();
-    if ((threadIdx.x & 31) == 0) mbar_arrive(bar);
-}
-
-// Producer warp of a staged CTA (the only mode-dependent code: row maps, fix-ups).
-// ntail > 0: the CTA's last ntail (= 2 HY) input rows -- the rows the next strip reads
-// first -- are fetched at the START into a dedicated buffer, while the neighbour strip
-// reads them too, so they come from DRAM once (L2) instead of once per strip.
-template <class Op, int MODE, int CK>
-__device__ __forceinline__ void staged_producer(const typename Op::Params &p, uint64_t *full, uint64_t *empty,
-                                                uint64_t *tailbar, typename Op::Tin *buf, typename Op::Tin *tail,
-                                                int ntail, int y0, int nr, int X0)
-{
-    using T = typename Op::Tin;
-    constexpr int HY = Op::HY, NIN = Op::NIN;
-    const Geom &g = p.g;
-    const int S = g.stages, SW = g.sw, RS = g.rs;
     const size_t row_elems = (size_t)NIN * SW, slot_elems = (size_t)RS * row_elems;
-    const int nhead = nr - ntail;
-    if (ntail > 0) {
-        for (int k = 0; k < ntail; ++k)
-            staged_fill_row<Op, MODE, CK>(p, tail + (size_t)k * row_elems, y0 - HY + nhead + k, X0, tailbar);
-        staged_fill_done<Op, MODE, CK>(p, tailbar);
-    }
-    // ---------------- ring: RS input rows per slot ----------------
+    // ---------------- producer warp: RS input rows per ring slot ----------------
     int s = 0, nfill = 0;
     uint32_t ph = 0;
-    for (int f0 = 0; f0 < nhead; f0 += RS, ++nfill) {
+    for (int f0 = 0; f0 < nr; f0 += RS, ++nfill) {
         if (nfill >= S) mbar_wait(&empty[s], ph ^ 1);
-        const int nrow = min(RS, nhead - f0);
+        const int nrow = min(RS, nr - f0);
         T *sb = buf + (size_t)s * slot_elems;
-        for (int k = 0; k < nrow; ++k)
-            staged_fill_row<Op, MODE, CK>(p, sb + (size_t)k * row_elems, y0 - HY + f0 + k, X0, &full[s]);
-        staged_fill_done<Op, MODE, CK>(p, &full[s]);
+        uint32_t bytes = 0;
+        for (int k = 0; k < nrow; ++k) {
+            bool rowok;
+            map_row<MODE, CK>(y0 - HY + f0 + k, g, rowok);
+            int cs = XS, ce = X0 + TW + HXA;
+            if constexpr ((CK & CK_L) != 0) cs = max(cs, 0);
+            if constexpr ((CK & CK_R) != 0) ce = min(ce, g.w_al);
+            if (!(MODE == CONSTANT && !rowok) && ce > cs) bytes += (uint32_t)(ce - cs) * (uint32_t)sizeof(T) * NIN;
+        }
+        if (lane == 0) mbar_expect_tx(&full[s], bytes);
+        for (int k = 0; k < nrow; ++k) {
+            bool rowok;
+            const int yy = map_row<MODE, CK>(y0 - HY + f0 + k, g, rowok);
+            int cs = XS, ce = X0 + TW + HXA;
+            if constexpr ((CK & CK_L) != 0) cs = max(cs, 0);
+            if constexpr ((CK & CK_R) != 0) ce = min(ce, g.w_al);
+            if (MODE == CONSTANT && !rowok) ce = cs;  // whole row = C
+            T *rb = sb + (size_t)k * row_elems;
+            if (lane == 0 && ce > cs)
+#pragma unroll
+                for (int c = 0; c < NIN; ++c)
+                    bulk_g2s(rb + (size_t)c * SW + (cs - XS), p.in[c] + (ptrdiff_t)yy * g.in_pitch + cs,
+                             (uint32_t)(ce - cs) * (uint32_t)sizeof(T), &full[s]);
+            if (CK != 0 && g.dbg != 4) {
+                // column fix-ups unless the compute warps rebuild the edge columns
+                const bool colfix = !((CK & (CK_L | CK_R)) && consumer_fix(g, PX));
+                // border fix-ups, this region's sides only (<= HXA columns per row):
+                // cp.async of the pattern's source column (4-byte types), else a
+                // synchronous copy; Constant: the constant
+#pragma unroll
+                for (int c = 0; c < NIN; ++c) {
+                    T *dst = rb + (size_t)c * SW;
+                    if (MODE == CONSTANT && !rowok) {
+                        for (int x = lane; x < SW; x += 32) dst[x] = p.cval;
+                        continue;
+                    }
+                    if (!colfix) continue;
+                    const T *src = p.in[c] + (ptrdiff_t)yy * g.in_pitch;
+                    auto fix = [&](int x) {
+                        if constexpr (MODE == CONSTANT) {
+                            dst[x - XS] = (x >= 0 && x < g.w) ? __ldg(src + x) : p.cval;
+                        } else {
+                            const int xs = fixup_source<Op, MODE, CK>(x, g);
+                            if (xs < 0) return;
+                            if constexpr (ASYNC_FIX) cp_async4(dst + (x - XS), src + xs);
+                            else dst[x - XS] = __ldg(src + xs);
+                        }
+                    };
+                    if constexpr ((CK & CK_L) != 0)
+                        for (int x = XS + lane; x < cs; x += 32) fix(x);
+                    if constexpr ((CK & CK_R) != 0)
+                        for (int x = ce + lane; x < X0 + TW + HXA; x += 32) fix(x);
+                }
+            }
+        }
+        if constexpr (ASYNC_FIX) {
+            if (g.dbg != 4 && !consumer_fix(g, PX)) cp_async_mbar_arrive_noinc(&full[s]);
+        }
+        if constexpr (MODE == CONSTANT && (CK & (CK_T | CK_B)) != 0)
+            fence_proxy_async();  // generic row fills before later bulk (async-proxy) writes
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&full[s]);
         if (++s == S) { s = 0; ph ^= 1; }
     }
 }
@@ -302,7 +277,6 @@ __device__ __forceinline__ void staged_body(const typename Op::Params &p, unsign
     const int S = g.stages, SW = g.sw, HXA = g.hxa;
     uint64_t *full = reinterpret_cast<uint64_t *>(smem);
     uint64_t *empty = full + kStagedMaxStages;
-    uint64_t *tailbar = empty + kStagedMaxStages;
     T *buf = reinterpret_cast<T *>(smem + kStagedBarrierBytes);
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     int y0, rows;
@@ -311,9 +285,6 @@ __device__ __forceinline__ void staged_body(const typename Op::Params &p, unsign
     const int X0 = blockIdx.x * TW;          // first output column of the CTA
     const int RS = g.rs;                     // rows per ring slot
     const size_t row_elems = (size_t)NIN * SW, slot_elems = (size_t)RS * row_elems;
-    const int ntail = g.tail ? 2 * HY : 0;   // last input rows, fetched first (staged_producer)
-    const int nhead = nr - ntail;
-    T *tail = buf + (size_t)S * slot_elems;
 
     // L/R CTAs of 4-byte types fetch their fix-up columns with cp.async: every producer
     // lane then arrives on the full barrier when its copies land (32 extra arrivals)
@@ -323,7 +294,6 @@ __device__ __forceinline__ void staged_body(const typename Op::Params &p, unsign
             mbar_init(&full[s], async_fix && g.dbg != 4 && !consumer_fix(g, Op::PX) ? 33 : 1);
             mbar_init(&empty[s], NWC);
         }
-        mbar_init(tailbar, async_fix && g.dbg != 4 && !consumer_fix(g, Op::PX) ? 33 : 1);
         fence_mbar_init();
     }
     __syncthreads();
@@ -332,10 +302,10 @@ __device__ __forceinline__ void staged_body(const typename Op::Params &p, unsign
 
     if (warp == NWC) {
         switch (g.mode) {  // the border pattern is a runtime parameter of the staged kernel
-        case CLAMP: staged_producer<Op, CLAMP, CK>(p, full, empty, tailbar, buf, tail, ntail, y0, nr, X0); break;
-        case MIRROR: staged_producer<Op, MIRROR, CK>(p, full, empty, tailbar, buf, tail, ntail, y0, nr, X0); break;
-        case REPEAT: staged_producer<Op, REPEAT, CK>(p, full, empty, tailbar, buf, tail, ntail, y0, nr, X0); break;
-        default: staged_producer<Op, CONSTANT, CK>(p, full, empty, tailbar, buf, tail, ntail, y0, nr, X0); break;
+        case CLAMP: staged_producer<Op, CLAMP, CK>(p, full, empty, buf, y0, nr, X0); break;
+        case MIRROR: staged_producer<Op, MIRROR, CK>(p, full, empty, buf, y0, nr, X0); break;
+        case REPEAT: staged_producer<Op, REPEAT, CK>(p, full, empty, buf, y0, nr, X0); break;
+        default: staged_producer<Op, CONSTANT, CK>(p, full, empty, buf, y0, nr, X0); break;
         }
         return;
     }
@@ -353,14 +323,8 @@ __device__ __forceinline__ void staged_body(const typename Op::Params &p, unsign
         for (int k = 0; k < MH; ++k) {
             const int r = r0 + k;
             if (r < nr) {
-                const bool from_tail = r >= nhead;
-                if (from_tail) {
-                    if (r == nhead) mbar_wait(tailbar, 0);
-                } else if (kr == 0) {
-                    mbar_wait(&full[s], ph);
-                }
-                const T *rb = from_tail ? tail + (size_t)(r - nhead) * row_elems
-                                        : buf + (size_t)s * slot_elems + (size_t)kr * row_elems;
+                if (kr == 0) mbar_wait(&full[s], ph);
+                const T *rb = buf + (size_t)s * slot_elems + (size_t)kr * row_elems;
                 RawRow<Op> rr;
                 if (g.dbg != 1) {
                     const T *srow[NIN];
@@ -368,7 +332,7 @@ __device__ __forceinline__ void staged_body(const typename Op::Params &p, unsign
                     for (int c = 0; c < NIN; ++c) srow[c] = rb + (size_t)c * SW + HXA + xoff;
                     load_row_smem<Op>(srow, rr);
                 }
-                if (!from_tail && (++kr == RS || r == nhead - 1)) {
+                if (++kr == RS || r == nr - 1) {
                     __syncwarp();
                     if (lane == 0) mbar_arrive(&empty[s]);  // release: the slot's rows are in registers
                     kr = 0;

@@ -25,6 +25,9 @@ struct Desc {
     float cval_f;
     int cval_i;
     int mw, mh;
+    int ax, ay;        // direct family: window anchor (cropped sparse masks, reading A31)
+    int reach[4];      // non-zero footprint reach L, R, T, B (has_reach)
+    int has_reach;
     const float *maskf, *rowf, *colf; // host
     const int *maski, *rowi, *coli;   // host
     U8RoundH rnd;

@@ -6,6 +6,7 @@ import ctypes
 import os
 import re
 
+import numpy as np
 import pytest
 
 import paper_conf_ipps_qiaoth21_b200 as isp
@@ -182,3 +183,34 @@ def test_model_form_s_matches_oracle():
                       threads_per_block=32)
         assert got["n_isp"] == pytest.approx(ref["N_ISP"], rel=1e-12)
         assert got["g"] == pytest.approx(ref["G"], rel=1e-12)
+
+
+# ---------------------------------------------------------------- N3: sparse masks (reading A31)
+def _sparse_masks(rng, n=40):
+    out = []
+    for _ in range(n):
+        m, k = int(rng.choice([3, 5, 7, 9, 13])), int(rng.choice([1, 3, 5, 7, 9]))
+        mask = np.where(rng.random((k, m)) < 0.4, rng.standard_normal((k, m)), 0.0)
+        mask[:, : int(rng.integers(0, m // 2 + 1))] = 0
+        mask[k - int(rng.integers(0, k // 2 + 1)):, :] = 0
+        out.append(mask)
+    return out
+
+
+def test_mask_reach_matches_oracle():
+    rng = np.random.default_rng(21)
+    for mask in _sparse_masks(rng):
+        assert isp.isp_mask_reach(mask.astype(np.float32)) == P.mask_reach(mask)
+        assert isp.isp_mask_reach(np.sign(mask).astype(np.int32)) == P.mask_reach(mask)
+
+
+def test_plan_reach_matches_oracle():
+    rng = np.random.default_rng(22)
+    for mask in _sparse_masks(rng):
+        r = P.mask_reach(mask)
+        for (w, h, tw, th) in [(4096, 4096, 512, 16), (300, 77, 128, 4), (40, 33, 32, 8)]:
+            got = isp.isp_plan_reach(w, h, r, tw, th)
+            b = P.bounds_reach(w, h, r, tw, th)
+            assert (got["bh_l"], got["bh_r"], got["bh_t"], got["bh_b"], got["nx"], got["ny"]) == \
+                (b["BH_L"], b["BH_R"], b["BH_T"], b["BH_B"], b["NX"], b["NY"])
+            assert bool(got["degenerate"]) == b["degenerate"]

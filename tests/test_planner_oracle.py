@@ -269,3 +269,51 @@ def test_model_form_s_closed_form():
     a = P.model(sx, sy, m, n, tx, ty, 0.0, k, form="S", threads_per_block=thr)
     b = P.model(sx, sy, m, n, tx, ty, 0.0, k, form="T", threads_per_block=thr)
     assert a["N_ISP"] == pytest.approx(b["N_ISP"], rel=1e-12)
+
+
+# ---------------------------------------------------------------- N3: sparse masks (reading A31)
+def test_mask_reach_examples():
+    m = np.zeros((7, 7))
+    m[3, 3] = 1
+    assert P.mask_reach(m) == (0, 0, 0, 0)
+    m[1, 5] = 2            # row 1 (2 above), column 5 (2 right)
+    assert P.mask_reach(m) == (0, 2, 2, 0)
+    m[6, 0] = -1           # row 6 (3 below), column 0 (3 left)
+    assert P.mask_reach(m) == (3, 2, 2, 3)
+    assert P.mask_reach(np.ones((5, 3))) == (1, 1, 2, 2)
+    assert P.mask_reach(np.zeros((3, 3))) == (0, 0, 0, 0)
+
+
+def test_bounds_reach_bruteforce():
+    """Eq. (2) from the non-zero footprint is conservative AND tight: per-thread
+    enumeration over the non-zero taps needs exactly the checks the bounds assign."""
+    rng = np.random.default_rng(11)
+    for _ in range(120):
+        m, n = int(rng.choice([3, 5, 7, 9])), int(rng.choice([1, 3, 5, 7]))
+        mask = (rng.random((n, m)) < 0.3).astype(float)
+        # zero edge rows / columns on purpose
+        if rng.random() < 0.5:
+            mask[:, : int(rng.integers(0, m // 2 + 1))] = 0
+        if rng.random() < 0.5:
+            mask[: int(rng.integers(0, n // 2 + 1)), :] = 0
+        sx, sy = int(rng.integers(6, 30)), int(rng.integers(6, 30))
+        tx, ty = int(rng.choice([2, 4, 8])), int(rng.choice([1, 2, 4]))
+        b = P.bounds_reach(sx, sy, P.mask_reach(mask), tx, ty)
+        if b["degenerate"]:
+            continue
+        for by in range(b["NY"]):
+            for bx in range(b["NX"]):
+                need = P.needed_sides_mask_bruteforce(sx, sy, mask, tx, ty, bx, by)
+                assert ("L" in need) == (bx < b["BH_L"])
+                assert ("R" in need) == (bx >= b["BH_R"])
+                assert ("T" in need) == (by < b["BH_T"])
+                assert ("B" in need) == (by >= b["BH_B"])
+
+
+def test_bounds_reach_dense_equals_eq2():
+    for (sx, sy, m, n, tx, ty) in [(512, 512, 13, 13, 32, 4), (100, 77, 7, 3, 16, 8), (4096, 4096, 5, 5, 512, 32)]:
+        hx, hy = m // 2, n // 2
+        a = P.bounds_reach(sx, sy, (hx, hx, hy, hy), tx, ty)
+        b = P.bounds(sx, sy, m, n, tx, ty)
+        assert {k: a[k] for k in ("BH_L", "BH_R", "BH_T", "BH_B", "NX", "NY", "degenerate")} == \
+               {k: b[k] for k in ("BH_L", "BH_R", "BH_T", "BH_B", "NX", "NY", "degenerate")}
