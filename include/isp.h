@@ -51,7 +51,13 @@ typedef enum { ISP_U8 = 0, ISP_I16 = 1, ISP_I32 = 2, ISP_F32 = 3 } isp_dtype_t;
  * checks only in the staging of border blocks, reading A21; needs 16-B aligned rows and
  * a compiled window, else runs as ISP_BLOCK); ISP_NAIVE = all four checks on every read
  * (Eq. 3 baseline). */
-typedef enum { ISP_AUTO = 0, ISP_BLOCK = 1, ISP_WARP = 2, ISP_NAIVE = 3, ISP_TMA = 4 } isp_variant_t;
+/* Ablations: ISP_SPLIT = one kernel per region (the nine regions launched
+ * separately over their block rectangles, instead of the paper's single fat kernel with
+ * the Listing-3 switch; plans like ISP_BLOCK); ISP_TEX = texture hardware border
+ * handling (every tap read through a texture object whose address mode implements
+ * the pattern -- clamp, mirror, wrap, border colour; isp_filter_ex only, 2-D FMA order). */
+typedef enum { ISP_AUTO = 0, ISP_BLOCK = 1, ISP_WARP = 2, ISP_NAIVE = 3, ISP_TMA = 4, ISP_SPLIT = 5,
+               ISP_TEX = 6 } isp_variant_t;
 typedef enum {
     ISP_OK = 0,
     ISP_EINVAL = 1,       /* bad size / pitch / window / mode / constant / divisor */

@@ -20,7 +20,8 @@ import os
 import torch
 
 __all__ = [
-    "CLAMP", "MIRROR", "REPEAT", "CONSTANT", "AUTO", "BLOCK", "WARP", "NAIVE", "TMA", "MODES", "VARIANTS",
+    "CLAMP", "MIRROR", "REPEAT", "CONSTANT", "AUTO", "BLOCK", "WARP", "NAIVE", "TMA", "SPLIT", "TEX", "MODES",
+    "VARIANTS",
     "lib", "IspError", "PlanInfo", "ModelParams",
     "isp_filter", "isp_filter_naive", "isp_filter_ex", "isp_filter_sep_f32", "isp_filter_u8",
     "isp_sobel_u8", "isp_laplace5_u8", "isp_harris_u8", "isp_pipeline_cfg3_u8", "isp_bilateral_f32", "isp_atrous_f32",
@@ -33,8 +34,8 @@ __all__ = [
 
 CLAMP, MIRROR, REPEAT, CONSTANT = 0, 1, 2, 3
 MODES = {"clamp": CLAMP, "mirror": MIRROR, "repeat": REPEAT, "constant": CONSTANT}
-AUTO, BLOCK, WARP, NAIVE, TMA = 0, 1, 2, 3, 4
-VARIANTS = {"auto": AUTO, "block": BLOCK, "warp": WARP, "naive": NAIVE, "tma": TMA}
+AUTO, BLOCK, WARP, NAIVE, TMA, SPLIT, TEX = 0, 1, 2, 3, 4, 5, 6
+VARIANTS = {"auto": AUTO, "block": BLOCK, "warp": WARP, "naive": NAIVE, "tma": TMA, "split": SPLIT, "tex": TEX}
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_HERE, "libisp.so")

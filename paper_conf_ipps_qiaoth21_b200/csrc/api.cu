@@ -308,14 +308,30 @@ int family_px(int fam, bool direct)
     }
 }
 
+// Model constants (reading A19), calibrated on B200 from ncu instruction counts
+// (profiles/r02_counters.json, tools/ncu_counters.py): per family and border mode, with I
+// = smsp__thread_inst_executed of one 4096^2 (Bilateral 2048^2) launch of px pixels,
+//   n_kernel = I_isp / (m n px)              (the ISP launch is essentially its Body)
+//   n_check  = (I_naive - I_isp) / (4 m n px)
+// i.e. instructions per tap of the computation and per border check per tap.  Families
+// in enum order F_CONV_F32 .. F_ATROUS; modes Clamp, Mirror, Repeat, Constant.
+const double kCalib[8][4][2] = {
+    {{0.1813, 1.7136}, {0.2368, 1.7221}, {0.5511, 1.6320}, {0.1120, 1.6949}},  // F_CONV_F32   (5x5 2-D)
+    {{0.1775, 0.8283}, {0.2475, 0.7370}, {0.5045, 0.8338}, {0.1129, 0.7146}},  // F_SEP_F32    (cfg2 5x5)
+    {{0.1534, 1.2677}, {0.2122, 1.2649}, {0.5123, 1.2502}, {0.2000, 1.2739}},  // F_U8         (5x5 Gaussian)
+    {{0.4532, 3.8122}, {0.5306, 3.8202}, {1.1165, 3.8433}, {0.4094, 3.8157}},  // F_SOBEL
+    {{0.1586, 0.9486}, {0.2288, 0.9393}, {0.4854, 0.9581}, {0.2037, 0.9316}},  // F_LAPLACE
+    {{0.7511, 6.3915}, {0.8680, 6.3961}, {2.2974, 6.4217}, {0.4643, 6.4138}},  // F_HARRIS
+    {{0.1995, 7.0678}, {0.3360, 7.1017}, {2.7004, 7.6321}, {0.6625, 7.2551}},  // F_BILATERAL  (13x13)
+    {{0.5936, 2.7106}, {0.6870, 2.7154}, {2.5672, 2.8571}, {0.6184, 2.7451}},  // F_ATROUS     (d = 2)
+};
+
 void defaults(int fam, int mode, isp_model_params &mp)
 {
-    // Calibration constants: instructions per border check per
-    // tap (mode-dependent) and per tap of the kernel computation.
-    static const double chk[4] = {1.0, 2.0, 3.0, 2.0};
-    mp.n_check = chk[mode & 3];
-    mp.n_kernel = fam == F_BILATERAL ? 8.0 : fam == F_HARRIS ? 3.0 : 1.0;
-    mp.ipc_switch = 2.0;
+    const int f = std::max(0, std::min(7, fam)), m = mode & 3;
+    mp.n_check = kCalib[f][m][0];
+    mp.n_kernel = kCalib[f][m][1];
+    mp.ipc_switch = 2.0;   // ISETP + BRA per Listing-3 compare (A18)
     mp.o_naive = -1;
     mp.o_isp = -1;
     mp.form = 0;
@@ -447,6 +463,9 @@ isp_status_t resolve_and_launch(Desc &d, int fam, int w, int h, int mw, int mh, 
                                 isp_variant_t v, KfnFn kfn, RunFn run, const char *what,
                                 const RowRange *rr = nullptr, bool tma_ok = false, int esz = 4, int nin = 1)
 {
+    if (v < ISP_AUTO || v > ISP_SPLIT)
+        return fail(v == ISP_TEX ? ISP_EUNSUPPORTED : ISP_EINVAL, "%s: variant %d%s", what, (int)v,
+                    v == ISP_TEX ? " (ISP_TEX: isp_filter_ex only)" : "");
     const int px = family_px(fam, direct);
     if (rr) {
         d.g.oy0 = rr->oy0;
@@ -489,7 +508,10 @@ isp_status_t resolve_and_launch(Desc &d, int fam, int w, int h, int mw, int mh, 
     if (use_p) nb_tma = std::min(nb_tma, pk.ctas);
     if (tma_ok && nb_tma <= 0) tma_ok = false;
 
-    isp_variant_t chosen = v;
+    // ISP_SPLIT (ablation of P:L90: one kernel per region instead of the fat kernel) plans
+    // like ISP_BLOCK and launches each region's block rectangle separately
+    const bool split = v == ISP_SPLIT;
+    isp_variant_t chosen = split ? ISP_BLOCK : v;
     if (chosen == ISP_TMA && !tma_ok) chosen = ISP_BLOCK;      // misaligned / not built: streaming
     // AUTO's ISP kernel: TMA-staged for 4-byte pixels; for sub-word pixels (u8, i16) the
     // staged L/R CTAs fix up their halo synchronously, so the streaming Listing-5 kernel
@@ -537,12 +559,8 @@ isp_status_t resolve_and_launch(Desc &d, int fam, int w, int h, int mw, int mh, 
         n_block(p, info.n_block);
         if (chosen == ISP_TMA) mp.form = 2;   // staged kernels: checks per staged element (A21)
         model(p, w, rr ? rr->nrows : h, mw, mh, mp, info);
-        // Eq. (10) picks ISP iff G > 1.  B200 calibration (reading A29): the
-        // u8 streaming fat kernels lose to naive below G ~ 2.4 (instruction-cache footprint
-        // of nine bodies, which the model does not count), so AUTO requires G > 2.4 there.
-        // isp_plan() keeps the paper's threshold (it is pinned against the oracle model).
-        const double g_star = (fam == F_U8 && chosen != ISP_TMA) ? 2.4 : 1.0;
-        if (!(info.g > g_star)) chosen = ISP_NAIVE;
+        // Eq. (10): ISP iff G > 1 (reading A20), with the calibrated constants (A19)
+        if (!(info.g > 1.0)) chosen = ISP_NAIVE;
     }
     if (chosen == ISP_NAIVE) p = plan_for(ISP_NAIVE);
     d.g.ty = p.ty;
@@ -584,6 +602,26 @@ isp_status_t resolve_and_launch(Desc &d, int fam, int w, int h, int mw, int mh, 
     if (const char *e = getenv("ISP_DEBUG_STAGED")) d.g.dbg = atoi(e);
     if (getenv("ISP_CTA_TRACE")) d.g.trace = cta_trace_buffer();
     d.g.edge_w = p.edge_w;
+    if (split && chosen == ISP_BLOCK) {
+        info.choice = ISP_SPLIT;
+        g_last_plan = info;
+        g_recent[g_n_plans++ % kRecent] = info;
+        const int cx[4] = {0, p.bh_l, p.bh_r, p.nx}, cy[4] = {0, p.bh_t, p.bh_b, p.ny};
+        static const int kReg[3][3] = {{RG_TL, RG_T, RG_TR}, {RG_L, RG_BODY, RG_R}, {RG_BL, RG_B, RG_BR}};
+        for (int rc = 0; rc < 3; ++rc)
+            for (int cc = 0; cc < 3; ++cc) {
+                if (cx[cc + 1] <= cx[cc] || cy[rc + 1] <= cy[rc]) continue;
+                Desc q = d;
+                q.grid = dim3(cx[cc + 1] - cx[cc], cy[rc + 1] - cy[rc], 1);
+                q.g.bx0 = cx[cc];
+                q.g.by0 = cy[rc];
+                q.g.force_rg = kReg[rc][cc];
+                cudaError_t e = run(q);
+                if (e == cudaSuccess) e = cudaGetLastError();
+                if (e != cudaSuccess) return cuda_status(e, what);
+            }
+        return ISP_OK;
+    }
     g_last_plan = info;
     g_recent[g_n_plans++ % kRecent] = info;
     cudaError_t e = run(d);
@@ -605,6 +643,7 @@ Desc base_desc(int w, int h, int pitch, int out_pitch, int mode, isp_stream_t st
     d.g.b_real = 1;
     d.mode = mode;
     d.stream = (cudaStream_t)stream;
+    d.g.force_rg = -1;
     return d;
 }
 
@@ -800,6 +839,10 @@ isp_status_t ispi_filter_f32(const float *img, int w, int h, int pitch, const fl
     if (!img || !out || !mask) return fail(ISP_EINVAL, "null pointer");
     if (!rr && ranges_overlap(img, img_bytes(w, h, pitch, 4), out, img_bytes(w, h, out_pitch, 4)))
         return fail(ISP_EALIAS, "input and output overlap");
+    if (variant == ISP_TEX) {   // ablation: texture-hardware border handling (texture.cu)
+        if (rr) return fail(ISP_EUNSUPPORTED, "ISP_TEX: row ranges (strips) not supported");
+        return ispi_filter_tex_f32(img, w, h, pitch, mask, mw, mh, border_mode, const_val, out, out_pitch, stream);
+    }
     Desc d = base_desc(w, h, pitch, out_pitch, border_mode, stream);
     d.in0 = img;
     d.out0 = out;

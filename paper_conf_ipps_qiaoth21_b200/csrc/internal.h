@@ -16,3 +16,5 @@ isp_status_t ispi_filter_f32(const float *img, int w, int h, int pitch, const fl
 isp_status_t ispi_filter_u8(const uint8_t *img, int w, int h, int pitch, const int32_t *mask, int mw, int mh,
                             int32_t divisor, int border_mode, int const_val, uint8_t *out, int out_pitch,
                             isp_variant_t variant, isp_stream_t stream, const RowRange *rr);
+isp_status_t ispi_filter_tex_f32(const float *img, int w, int h, int pitch, const float *mask, int mw, int mh,
+                                 int border_mode, float const_val, float *out, int out_pitch, isp_stream_t stream);

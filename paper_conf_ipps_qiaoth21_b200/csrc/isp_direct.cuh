@@ -66,7 +66,9 @@ __global__ void __launch_bounds__(256) k_direct(const __grid_constant__ typename
     const int lane = threadIdx.x & 31;
     const int warp = threadIdx.x >> 5;
     const int nwarp = blockDim.x >> 5;
-    const int bx = blockIdx.x, by = blockIdx.y;
+    // split launches (variant ISP_SPLIT, one kernel per region, P:L90 ablation): the
+    // launch covers one region's block rectangle starting at (bx0, by0)
+    const int bx = blockIdx.x + p.g.bx0, by = blockIdx.y + p.g.by0;
     const int gw = bx * nwarp + warp;
     const int x0 = (gw * 32 + lane) * Op::PX;
     int y0, rows;
@@ -76,7 +78,7 @@ __global__ void __launch_bounds__(256) k_direct(const __grid_constant__ typename
     } else if constexpr (DISP == DISP_NAIVE_GEN) {
         direct_body<Op, MODE, CK_ALL | CK_GEN>(p, x0, y0, rows);
     } else {
-        const int rg = region_of(p.g, bx, by, gw, p.g.warp_level != 0);
+        const int rg = p.g.force_rg >= 0 ? p.g.force_rg : region_of(p.g, bx, by, gw, p.g.warp_level != 0);
         switch (rg) {
         case RG_TL: direct_body<Op, MODE, region_checks(RG_TL)>(p, x0, y0, rows); break;
         case RG_TR: direct_body<Op, MODE, region_checks(RG_TR)>(p, x0, y0, rows); break;

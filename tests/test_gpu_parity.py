@@ -357,19 +357,17 @@ def test_strips_local_equal_full_image(isp, nranks, m):
             np.testing.assert_array_equal(got, ref, err_msg=f"{mode} {v} P={nranks}")
 
 
-def test_auto_u8_calibrated_threshold(isp):
-    """Reading A29: launch-time AUTO takes the u8 streaming ISP kernel only when G > 2.4
-    (the measured B200 crossover), while isp_plan() keeps the paper's G > 1; results
-    stay identical to the oracle either way."""
+def test_auto_follows_eq10(isp):
+    """AUTO ("isp+m") takes the ISP kernel iff the model's G > 1 (Eq. 10, reading A20) with
+    the B200-calibrated constants (A19, profiles/r02_counters.json) -- no other threshold;
+    results identical to the oracle either way."""
     g5 = np.outer(synth.binomial_row(5), synth.binomial_row(5)).astype(np.int32)
-    for n in (1024, 4096):
+    for n in (512, 1024, 4096):
         img = synth.structured_u8(n, n, 3)
         out = isp.isp_filter_u8(dev(img), g5, int(g5.sum()), "clamp", 7)
         torch.cuda.synchronize()
         plan = isp.isp_last_plan()
-        if plan["g"] > 2.4:
-            assert plan["choice"] != 3, plan
-        elif not plan["degenerate"]:
-            assert plan["choice"] == 3, plan
+        if not plan["degenerate"]:
+            assert (plan["choice"] != 3) == (plan["g"] > 1.0), plan
         rows = sample_rows(n, k=4, seed=n)
         np.testing.assert_array_equal(host(out)[rows], oracle.filter_u8(img, g5, int(g5.sum()), "clamp", 7, rows=rows))

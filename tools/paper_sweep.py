@@ -28,10 +28,11 @@ import torch  # noqa: E402
 
 import paper_conf_ipps_qiaoth21_b200 as isp  # noqa: E402
 import synth  # noqa: E402
-from bench_suite import nbuf_for, time_launch  # noqa: E402
+from bench_suite import binomial_f32, nbuf_for, time_launch  # noqa: E402
 
 MODES = ["clamp", "mirror", "repeat", "constant"]
-VARIANTS = ["naive", "warp", "block", "tma", "auto"]
+VARIANTS = ["naive", "warp", "block", "tma", "split", "tex", "auto"]
+CHOOSABLE = ["naive", "warp", "block", "tma"]       # what AUTO can pick; split / tex are ablations
 SIZES = [512, 1024, 2048, 4096]
 G5 = np.outer(synth.binomial_row(5), synth.binomial_row(5)).astype(np.int32)
 
@@ -44,7 +45,10 @@ def app_fns(n):
     def f32_in():
         return torch.from_numpy(synth.structured_f32(n, n, 4)).cuda()
 
+    g5f = binomial_f32(5)
     return [
+        ("gaussian_f32_5x5", 8, lambda: (f32_in(), torch.empty((n, n), dtype=torch.float32, device="cuda")),
+         lambda b, m, v: isp.isp_filter_ex(b[0], g5f, m, 0.5, out=b[1], variant=v)),
         ("gaussian_u8_5x5", 2, lambda: (u8_in(), torch.empty((n, n), dtype=torch.uint8, device="cuda")),
          lambda b, m, v: isp.isp_filter_u8(b[0], G5, int(G5.sum()), m, 7, out=b[1], variant=v)),
         ("laplace5_u8", 2, lambda: (u8_in(), torch.empty((n, n), dtype=torch.uint8, device="cuda")),
@@ -75,8 +79,16 @@ def geo(xs):
     return math.exp(sum(math.log(x) for x in xs) / len(xs)) if xs else None
 
 
+def pearson(xs, ys):
+    xs, ys = np.asarray(xs, float), np.asarray(ys, float)
+    if len(xs) < 3 or xs.std() == 0 or ys.std() == 0:
+        return None
+    return float(np.corrcoef(xs, ys)[0, 1])
+
+
 def main():
     out = {"device": torch.cuda.get_device_name(0), "apps": {}, "geomean": {}}
+    match, cells = 0, 0
     for n in SIZES:
         for name, bpp, make, launch in app_fns(n):
             nb = nbuf_for(bpp * n * n)
@@ -87,25 +99,60 @@ def main():
                 isp_us = [r[v]["us"] for v in ("warp", "block", "tma") if "us" in r[v]]
                 r["speedup_best_isp"] = base / min(isp_us) if base and isp_us else None
                 r["speedup_auto"] = base / r["auto"]["us"] if base and "us" in r["auto"] else None
+                best = min(r[v]["us"] for v in CHOOSABLE if "us" in r[v])
+                r["auto_matches_best"] = bool(r["auto"].get("us", 1e30) <= 1.05 * best)
+                match += r["auto_matches_best"]
+                cells += 1
                 out["apps"].setdefault(name, {}).setdefault(str(n), {})[mode] = r
             del bufs
             torch.cuda.empty_cache()
         print(f"[sweep] {n} done", file=sys.stderr, flush=True)
+    out["auto_matches_best_within_5pct"] = {"cells": cells, "matches": match, "rate": match / max(cells, 1)}
     for name, per in out["apps"].items():
         best = [per[s][m]["speedup_best_isp"] for s in per for m in per[s]]
         auto = [per[s][m]["speedup_auto"] for s in per for m in per[s]]
         out["geomean"][name] = {"best_isp_vs_naive": geo(best), "auto_vs_naive": geo(auto),
                                 "min_auto_vs_naive": min(a for a in auto if a), "n": len(auto)}
-    # Table III / Fig. 4 analog: Gaussian size sweep, clamp, ISP (auto) vs naive
+    # Table III / Fig. 4 analog: Bilateral 13x13, image sizes 512..4096 step
+    # 256, per border pattern: measured speedup of the direct Listing-3 ISP kernel over
+    # naive vs the model's G for that launch (Eq. 10, calibrated constants), Pearson r.
+    t3 = {}
+    for mode in MODES:
+        rows = []
+        for n in range(512, 4097, 256):
+            f = torch.from_numpy(synth.structured_f32(n, n, 4)).cuda()
+            nb = nbuf_for(8 * n * n)
+            bufs = [(f, torch.empty_like(f)) for _ in range(nb)]
+
+            def lb(b, m, v):
+                return isp.isp_bilateral_f32(b[0], 13, 3.0, 0.1, m, 0.5, out=b[1], variant=v)
+            tn = time_app(n, 8, None, lb, mode, "naive", bufs)
+            tb = time_app(n, 8, None, lb, mode, "block", bufs)
+            ta = time_app(n, 8, None, lb, mode, "auto", bufs)
+            lb(bufs[0], mode, "block")
+            pb = isp.isp_last_plan()
+            gb = isp.isp_plan(n, n, 13, 13, tile_w=pb["tile_w"], tile_h=pb["tile_h"], warp_w=pb["warp_w"],
+                              border_mode=mode, filter_id=6)["g"]
+            rows.append({"n": n, "naive_us": tn["us"], "block_us": tb["us"], "auto_us": ta["us"],
+                         "speedup_block": tn["us"] / tb["us"], "speedup_auto": tn["us"] / ta["us"],
+                         "G_block": gb, "G_auto": ta["G"], "auto_choice": ta["choice"]})
+            del bufs, f
+            torch.cuda.empty_cache()
+        t3[mode] = {"rows": rows,
+                    "pearson_G_vs_speedup_block": pearson([r["G_block"] for r in rows], [r["speedup_block"] for r in rows]),
+                    "pearson_G_vs_speedup_auto": pearson([r["G_auto"] for r in rows], [r["speedup_auto"] for r in rows])}
+        print(f"[sweep] table III {mode} done", file=sys.stderr, flush=True)
+    out["table3_bilateral13"] = t3
+    # Gaussian u8 size sweep, clamp, AUTO vs naive
     sweep = {}
     for n in range(512, 4097, 256):
-        name, bpp, make, launch = app_fns(n)[0]
+        name, bpp, make, launch = app_fns(n)[1]
         nb = nbuf_for(bpp * n * n)
         bufs = [make() for _ in range(nb)]
-        sweep[str(n)] = {v: time_app(n, bpp, make, launch, "clamp", v, bufs) for v in ("naive", "auto")}
+        sweep[str(n)] = {v: time_app(n, bpp, make, launch, "clamp", v, bufs) for v in ("naive", "warp", "auto")}
         sweep[str(n)]["speedup_auto"] = sweep[str(n)]["naive"]["us"] / sweep[str(n)]["auto"]["us"]
         del bufs
-    out["gaussian_size_sweep_clamp"] = sweep
+    out["gaussian_u8_size_sweep_clamp"] = sweep
     print(json.dumps(out, indent=1))
 
 
