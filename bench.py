@@ -307,10 +307,32 @@ def run_isp(args):
         ctx = isp.isp_shard_init(uid[0], rank, world, local)
     stream = torch.cuda.Stream(device=dev)
     variant = args.variant
+    # N > 1 halo path: "peer" (default) -- every rank reads its neighbours' edge rows straight
+    # from their strips over NVLink (CUDA IPC), one launch per rank and mode, no exchange;
+    # "nccl" -- halo rows exchanged with NCCL send/recv, then the edge rows launched.
+    halo_path = args.halo if world > 1 else None
+    peers = None
+    if world > 1 and halo_path == "peer":
+        try:
+            own = [pairs[k][0][halo:halo + sh] for k in range(npairs)]
+            peers = [isp.isp_shard_peer_open(ctx, o, ring=True) for o in own]
+            ok = torch.tensor([1.0], device=dev)
+        except Exception as e:   # no IPC in this environment: fall back to the NCCL exchange
+            print(f"[bench] rank {rank}: peer open failed ({e}); using the NCCL halo exchange", file=sys.stderr)
+            ok = torch.tensor([0.0], device=dev)
+        dist.all_reduce(ok, op=dist.ReduceOp.MIN)
+        if ok.item() < 1:
+            if peers:
+                for pp in peers:
+                    isp.isp_shard_peer_close(pp)
+            peers, halo_path = None, "nccl (peer open failed)"
+        dist.barrier()      # every strip holds its data before any rank reads a neighbour's
 
     def launch(mode, pair, v=variant):
         inp, out = pairs[pair]
-        if world > 1:
+        if world > 1 and peers is not None:
+            isp.isp_shard_peer_filter_f32(peers[pair], H_img, mask, mode, CONST, out=out, variant=v, stream=stream)
+        elif world > 1:
             isp.isp_shard_filter_f32(ctx, inp, H_img, halo, mask, mode, CONST, out=out, variant=v, stream=stream,
                                      comm_stream=comm_stream)
         else:
@@ -320,7 +342,9 @@ def run_isp(args):
         for i, m in enumerate(modes):
             launch(m, (nm * k + i) % npairs, v)
 
-    if world > 1:
+    if world > 1 and peers is not None:
+        launches_per_step = nm
+    elif world > 1:
         launches_per_step = sum(len([l for l in isp.isp_shard_schedule(H_img, rank, world, halo, halo,
                                                                        isp.MODES[m])["launch"] if l[1] > 0])
                                 for m in modes)
@@ -505,6 +529,11 @@ def run_isp(args):
     if rank == 0 and world == 1 and not args.no_cpu:
         cpu = cpu_oracle_rate(workload=wl)
 
+    if peers is not None:
+        torch.cuda.synchronize()
+        dist.barrier()
+        for pp in peers:
+            isp.isp_shard_peer_close(pp)
     if ctx is not None:
         torch.cuda.synchronize()
         isp.isp_shard_destroy(ctx)
@@ -513,8 +542,8 @@ def run_isp(args):
                 "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True, "scaling": wl.scaling,
                 "vs_baseline": None, "dtype": "f32", "data": "synthetic",
                 "config": {"workload": wl.desc
-                                       + (f"; {world} ranks = row strips of the {H_img}x{W} image, NCCL halo "
-                                          "exchange" if world > 1 else ""),
+                                       + (f"; {world} ranks = row strips of the {H_img}x{W} image, halo rows "
+                                          f"via {halo_path}" if world > 1 else ""),
                            "image": [H_img, W], "window": [wl.window, wl.window], "const": CONST,
                            "modes": modes,
                            "l2": f"rotating {npairs} in/out buffer pairs "
@@ -527,8 +556,10 @@ def run_isp(args):
                 "gpu_launches": args.steps * launches_per_step, "clocks": clocks,
                 "isp_vs_naive": variants or None}
         if world > 1:
+            line["halo_path"] = halo_path
             line["halo_exchange_us"] = halo_us
             line["per_rank_rows"] = sh
+            line["config"]["halo"] = halo_path
         print(json.dumps(line), flush=True)
     if world > 1:
         dist.destroy_process_group()
@@ -582,6 +613,8 @@ def main():
                     help="cfg2: BASELINE configs[1] (default, weak scaling over ranks); "
                          "cfg5: configs[4] 16384^2 7x7 strong scaling")
     ap.add_argument("--check-launch", action="store_true", help="only check the N-rank launch path")
+    ap.add_argument("--halo", default="peer", choices=["peer", "nccl"],
+                    help="N > 1: neighbour rows read from peer memory (default) or exchanged with NCCL")
     ap.add_argument("--steps", type=int, default=6000)
     ap.add_argument("--warmup", type=int, default=20)
     ap.add_argument("--impl", default="isp", choices=["isp", "reference"])

@@ -260,6 +260,35 @@ isp_status_t isp_shard_filter_local_f32(float *strip, int w, int H, int pitch, i
  * and for callers that run their own launches.  Stream-ordered; no filtering. */
 isp_status_t isp_shard_exchange(isp_shard_ctx *ctx, void *strip, int elem_size, int H, int pitch, int halo, int hy,
                                 int border_mode, isp_stream_t comm_stream);
+/* Peer-direct strips: each rank's `strip` holds ONLY its own strip_h rows
+ * (pitch elements each, no halo rows); the hy rows above / below are read straight from the
+ * neighbour ranks' strips in peer memory (CUDA IPC mappings over NVLink), so one launch
+ * covers the strip and no halo exchange runs.  Only rank 0 / P-1 own the image T / B
+ * borders (Repeat: the ring neighbours supply the wrapped rows).
+ *   isp_shard_peer_open: collective over the ctx's ranks (NCCL all-gather of the IPC
+ *     handles of every rank's strip allocation); ring != 0 also maps the wrap neighbours
+ *     (needed for Repeat).  The strip must stay allocated until isp_shard_peer_close.
+ *   Ordering contract: every rank's strip must hold its data before any rank's filter
+ *     call starts (e.g. a process-group barrier after writing them) and must not be
+ *     rewritten until the neighbours' calls have finished.
+ *   isp_shard_filter_peer_local_*: the same launch with explicit neighbour pointers
+ *     (prev = rank r-1's strip, next = rank r+1's, ring neighbours for Repeat at the ends;
+ *     any pointers the device can read -- single-GPU emulation in tests).
+ * f32 and u8 filters (isp_filter_ex / isp_filter_u8 semantics, all variants except TEX). */
+typedef struct isp_shard_peer isp_shard_peer;
+isp_status_t isp_shard_peer_open(isp_shard_ctx *ctx, void *strip, int ring, isp_shard_peer **out);
+isp_status_t isp_shard_peer_filter_f32(isp_shard_peer *peer, int w, int H, int pitch, const float *mask, int mw,
+                                       int mh, int border_mode, float const_val, float *out, int out_pitch,
+                                       isp_variant_t variant, isp_stream_t stream);
+isp_status_t isp_shard_peer_close(isp_shard_peer *peer);
+isp_status_t isp_shard_filter_peer_local_f32(const float *own, const float *prev, const float *next, int w, int H,
+                                             int pitch, int rank, int nranks, const float *mask, int mw, int mh,
+                                             int border_mode, float const_val, float *out, int out_pitch,
+                                             isp_variant_t variant, isp_stream_t stream);
+isp_status_t isp_shard_filter_peer_local_u8(const uint8_t *own, const uint8_t *prev, const uint8_t *next, int w,
+                                            int H, int pitch, int rank, int nranks, const int32_t *mask, int mw,
+                                            int mh, int32_t divisor, int border_mode, int const_val, uint8_t *out,
+                                            int out_pitch, isp_variant_t variant, isp_stream_t stream);
 /* u8 counterpart of isp_shard_filter_local_f32 (the launch part of isp_shard_filter_u8). */
 isp_status_t isp_shard_filter_local_u8(uint8_t *strip, int w, int H, int pitch, int halo, int rank, int nranks,
                                        const int32_t *mask, int mw, int mh, int32_t divisor, int border_mode,

@@ -29,7 +29,8 @@ __all__ = [
     "isp_set_launch_override",
     "isp_shard_unique_id", "isp_shard_init", "isp_shard_rows", "isp_shard_schedule",
     "isp_shard_filter_f32", "isp_shard_filter_u8", "isp_shard_filter_local_f32", "isp_shard_filter_local_u8",
-    "isp_shard_exchange", "isp_shard_destroy",
+    "isp_shard_exchange", "isp_shard_destroy", "isp_shard_peer_open", "isp_shard_peer_filter_f32",
+    "isp_shard_peer_close", "isp_shard_filter_peer_local_f32", "isp_shard_filter_peer_local_u8",
 ]
 
 CLAMP, MIRROR, REPEAT, CONSTANT = 0, 1, 2, 3
@@ -118,6 +119,12 @@ _SIGS = {
     "isp_recent_plans": [_P, _I],
     "isp_shard_exchange": [_P, _P, _I, _I, _I, _I, _I, _I, _P],
     "isp_mask_reach": [_P, _I, _I, _I, _P],
+    "isp_shard_peer_open": [_P, _P, _I, _P],
+    "isp_shard_peer_filter_f32": [_P, _I, _I, _I, _P, _I, _I, _I, _F, _P, _I, _I, _P],
+    "isp_shard_peer_close": [_P],
+    "isp_shard_filter_peer_local_f32": [_P, _P, _P, _I, _I, _I, _I, _I, _P, _I, _I, _I, _F, _P, _I, _I, _P],
+    "isp_shard_filter_peer_local_u8": [_P, _P, _P, _I, _I, _I, _I, _I, _P, _I, _I, ctypes.c_int32, _I, _I, _P, _I,
+                                       _I, _P],
     "isp_plan_reach": [_I, _I, _P, _I, _I, _I, _P],
 }
 
@@ -528,6 +535,73 @@ def isp_shard_exchange(ctx, strip, H, halo, hy, border_mode, comm_stream=None, r
     cs = comm_stream if comm_stream is not None else torch.cuda.current_stream(strip.device)
     _check(lib().isp_shard_exchange(ctx, strip.data_ptr(), strip.element_size(), int(H), strip.shape[1], int(halo),
                                     int(hy), _mode(border_mode), ctypes.c_void_p(cs.cuda_stream)))
+
+
+def _own_strip(strip, dtype, H, rank, nranks, name="strip"):
+    _img(strip, dtype, name)
+    _, sh = isp_shard_rows(H, rank, nranks)
+    if strip.shape[0] != sh:
+        raise ValueError(f"peer {name} has {strip.shape[0]} rows, rank {rank}/{nranks} of H={H} owns {sh}")
+    return sh
+
+
+def isp_shard_filter_peer_local_f32(own, prev, nxt, H, rank, nranks, mask, border_mode, const_val=0.0, out=None,
+                                    variant=AUTO, w=None, stream=None):
+    """Peer-direct strip launch (no halo rows): neighbour rows read from prev / nxt strips."""
+    sh = _own_strip(own, torch.float32, H, rank, nranks)
+    w, _, pitch = _geom(own, w)
+    m, mp = _host(mask, ctypes.c_float)
+    mh, mw = m.shape
+    out = _out(out, own, w, torch.float32, rows=sh)
+    ptr = lambda t: t.data_ptr() if t is not None else None  # noqa: E731
+    _check(lib().isp_shard_filter_peer_local_f32(own.data_ptr(), ptr(prev), ptr(nxt), w, int(H), pitch, int(rank),
+                                                 int(nranks), mp, mw, mh, _mode(border_mode), float(const_val),
+                                                 out.data_ptr(), out.shape[1], _variant(variant), _stream(own, stream)))
+    return out
+
+
+def isp_shard_filter_peer_local_u8(own, prev, nxt, H, rank, nranks, mask, divisor, border_mode, const_val=0, out=None,
+                                   variant=AUTO, w=None, stream=None):
+    sh = _own_strip(own, torch.uint8, H, rank, nranks)
+    w, _, pitch = _geom(own, w)
+    m, mp = _host(mask, ctypes.c_int32)
+    mh, mw = m.shape
+    out = _out(out, own, w, torch.uint8, rows=sh)
+    ptr = lambda t: t.data_ptr() if t is not None else None  # noqa: E731
+    _check(lib().isp_shard_filter_peer_local_u8(own.data_ptr(), ptr(prev), ptr(nxt), w, int(H), pitch, int(rank),
+                                                int(nranks), mp, mw, mh, int(divisor), _mode(border_mode),
+                                                int(const_val), out.data_ptr(), out.shape[1], _variant(variant),
+                                                _stream(own, stream)))
+    return out
+
+
+def isp_shard_peer_open(ctx, strip, ring=True):
+    """Collective: map the neighbour ranks' strips (CUDA IPC); strip = own rows only."""
+    pp = ctypes.c_void_p()
+    _check(lib().isp_shard_peer_open(ctx, strip.data_ptr(), int(bool(ring)), ctypes.byref(pp)))
+    _PEER_CTX[pp.value] = (ctx, strip)
+    return pp
+
+
+_PEER_CTX = {}
+
+
+def isp_shard_peer_filter_f32(pp, H, mask, border_mode, const_val=0.0, out=None, variant=AUTO, w=None, stream=None):
+    ctx, strip = _PEER_CTX[pp.value]
+    rank, nranks = _ctx_ranks(ctx, None, None)
+    sh = _own_strip(strip, torch.float32, H, rank, nranks)
+    w, _, pitch = _geom(strip, w)
+    m, mp = _host(mask, ctypes.c_float)
+    mh, mw = m.shape
+    out = _out(out, strip, w, torch.float32, rows=sh)
+    _check(lib().isp_shard_peer_filter_f32(pp, w, int(H), pitch, mp, mw, mh, _mode(border_mode), float(const_val),
+                                           out.data_ptr(), out.shape[1], _variant(variant), _stream(strip, stream)))
+    return out
+
+
+def isp_shard_peer_close(pp):
+    _PEER_CTX.pop(pp.value, None)
+    _check(lib().isp_shard_peer_close(pp))
 
 
 def isp_shard_destroy(ctx):

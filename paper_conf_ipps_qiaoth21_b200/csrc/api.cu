@@ -158,10 +158,14 @@ Plan make_plan(int w, int h, int hx, int hy, int px, int tile_w_req, int tile_h_
     p.w_l = (int)ceil_div(hx, warp_w);
     p.w_r = (int)floor_div(w - hxr, warp_w);
     // Eq. (2) in y, relative to the launch's first row oy0; only real image edges count.
+    // a peer strip's edges are region edges as well (rows beyond them live in another
+    // buffer): top edge at own_y0, bottom edge at own_y1 (reading of SURVEY 8(f) N4)
+    const bool pt = rr->peer && !rr->t_real, pb = rr->peer && !rr->b_real;
+    const long long top_edge = rr->t_real ? 0 : rr->own_y0, bot_edge = rr->b_real ? h : rr->own_y1;
     if (p.ty > 0) {
-        p.bh_t = rr->t_real ? (int)std::max<long long>(0, ceil_div(hy - rr->oy0, p.ty)) : 0;
-        const long long safe_end = rr->b_real ? std::min<long long>(rr->oy0 + nr, (long long)h - hyb)
-                                              : rr->oy0 + nr;
+        p.bh_t = (rr->t_real || pt) ? (int)std::max<long long>(0, ceil_div(hy - (rr->oy0 - top_edge), p.ty)) : 0;
+        const long long safe_end = (rr->b_real || pb) ? std::min<long long>(rr->oy0 + nr, bot_edge - hyb)
+                                                      : rr->oy0 + nr;
         p.bh_b = (int)floor_div(safe_end - rr->oy0, p.ty);
     } else {
         // same definition on the balanced split: first block row whose reads stay >= 0,
@@ -176,11 +180,11 @@ Plan make_plan(int w, int h, int hx, int hy, int px, int tile_w_req, int tile_h_
             return rr->oy0 + (c * nr) / W;
         };
         int bt = 0;
-        if (rr->t_real)
-            while (bt < p.ny && y0_of(bt) - hy < 0) ++bt;
+        if (rr->t_real || pt)
+            while (bt < p.ny && y0_of(bt) - hy < top_edge) ++bt;
         int bb = p.ny;
-        if (rr->b_real)
-            while (bb > 0 && y0_of(bb) + hyb > h) --bb;   // y0_of(bb) = end of block bb-1
+        if (rr->b_real || pb)
+            while (bb > 0 && y0_of(bb) + hyb > bot_edge) --bb;   // y0_of(bb) = end of block bb-1
         p.bh_t = bt;
         p.bh_b = bb;
         if (bt <= bb) {
@@ -473,6 +477,11 @@ isp_status_t resolve_and_launch(Desc &d, int fam, int w, int h, int mw, int mh, 
         d.g.ylim = rr->ylim;
         d.g.t_real = rr->t_real;
         d.g.b_real = rr->b_real;
+        d.g.peer = rr->peer;
+        d.g.own_y0 = rr->own_y0;
+        d.g.own_y1 = rr->own_y1;
+        d.g.peer_lo = rr->peer_lo;
+        d.g.peer_hi = rr->peer_hi;
     }
     // reaches of the window (left, right, top, bottom): the non-zero footprint of a
     // cropped sparse mask (reading A31), else hx / hy on both sides

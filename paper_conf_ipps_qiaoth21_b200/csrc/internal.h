@@ -5,8 +5,14 @@
 // Output row range of a launch: rows [oy0, oy0+nrows) of an image of height h whose
 // resident input rows end at ylim; t_real / b_real: the range's top / bottom edge is a
 // real image edge (else a strip edge whose neighbour rows arrive by halo exchange).
+// peer (peer-direct halos): the strip's own rows are [own_y0, own_y1) of
+// the buffer `img` points into; rows above / below come straight from the neighbour
+// strips' memory (peer_lo / peer_hi, global-row addressed like img) -- the strip edges are
+// then region edges too (their block rows select the neighbour buffer per row).
 struct RowRange {
     int oy0, nrows, ylim, t_real, b_real;
+    int peer = 0, own_y0 = 0, own_y1 = 0;
+    const void *peer_lo = nullptr, *peer_hi = nullptr;
 };
 
 isp_status_t ispi_fail(isp_status_t s, const char *fmt, ...);

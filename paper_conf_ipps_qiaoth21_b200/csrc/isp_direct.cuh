@@ -42,7 +42,7 @@ __device__ __forceinline__ void direct_body(const typename Op::Params &p, int x0
         for (int j = 0; j < p.mh; ++j) {
             bool rowok;
             const int yy = map_row<MODE, CK>(y + j - hy, g, rowok);
-            const T *__restrict__ row = p.in + (ptrdiff_t)yy * g.in_pitch;
+            const T *__restrict__ row = row_base<CK>(p.in, yy, g);
             T win[PX];
 #pragma unroll
             for (int e = 0; e < PX; ++e) win[e] = load_x<T, MODE, CK>(row, rowok, x0 - hx + e, g, p.cval);
@@ -116,7 +116,7 @@ __device__ __forceinline__ void tile_fill(const typename Op::Params &p, typename
     for (int r = threadIdx.x / 32; r < SH; r += kTileWarps) {
         bool rowok;
         const int yy = map_row<MODE, CK>(Y0 - hy + r, g, rowok);
-        const T *__restrict__ row = p.in + (ptrdiff_t)yy * g.in_pitch;
+        const T *__restrict__ row = row_base<CK>(p.in, yy, g);
         T *dst = tile + r * SW;
         for (int c = threadIdx.x & 31; c < SW; c += 32) {
             const int x = X0 - hx + c;

@@ -88,7 +88,7 @@ __device__ __forceinline__ void pstaged_produce(const typename Op::Params &p, ui
             const T *const *in = p.in;
 #pragma unroll
             for (int c = 0; c < NIN; ++c) {
-                const T *src = in[c] + (ptrdiff_t)yy * g.in_pitch;
+                const T *src = row_base<CK>(in[c], yy, g);
                 T *dst = rb + (size_t)c * SW;
                 if (ce > cs) bulk_g2s(dst + (cs - XS), src + cs, (uint32_t)(ce - cs) * (uint32_t)sizeof(T), &full[s]);
                 if (wl) bulk_g2s(dst, src + g.w - wl, (uint32_t)wl * (uint32_t)sizeof(T), &full[s]);
@@ -104,7 +104,7 @@ __device__ __forceinline__ void pstaged_produce(const typename Op::Params &p, ui
                     continue;
                 }
                 if (!colfix || rep_bulk) continue;
-                const T *src = p.in[c] + (ptrdiff_t)yy * g.in_pitch;
+                const T *src = row_base<CK>(p.in[c], yy, g);
                 auto fix = [&](int x) {
                     if constexpr (MODE == CONSTANT) {
                         dst[x - XS] = (x >= 0 && x < g.w) ? __ldg(src + x) : p.cval;

@@ -222,7 +222,7 @@ __device__ __forceinline__ void staged_producer(const typename Op::Params &p, ui
             if (lane == 0 && ce > cs)
 #pragma unroll
                 for (int c = 0; c < NIN; ++c)
-                    bulk_g2s(rb + (size_t)c * SW + (cs - XS), p.in[c] + (ptrdiff_t)yy * g.in_pitch + cs,
+                    bulk_g2s(rb + (size_t)c * SW + (cs - XS), row_base<CK>(p.in[c], yy, g) + cs,
                              (uint32_t)(ce - cs) * (uint32_t)sizeof(T), &full[s]);
             if (CK != 0 && g.dbg != 4) {
                 // column fix-ups unless the compute warps rebuild the edge columns
@@ -238,7 +238,7 @@ __device__ __forceinline__ void staged_producer(const typename Op::Params &p, ui
                         continue;
                     }
                     if (!colfix) continue;
-                    const T *src = p.in[c] + (ptrdiff_t)yy * g.in_pitch;
+                    const T *src = row_base<CK>(p.in[c], yy, g);
                     auto fix = [&](int x) {
                         if constexpr (MODE == CONSTANT) {
                             dst[x - XS] = (x >= 0 && x < g.w) ? __ldg(src + x) : p.cval;

@@ -12,11 +12,13 @@
 //   exchange; launches 1/2 (after the halo event): the hy rows at each halo edge.
 // Only rank 0 owns the image's T border and rank P-1 its B border (Clamp, Mirror,
 // Constant); interior ranks run only L / Body / R regions.
+#include <cuda.h>
 #include <cuda_runtime.h>
 #include <nccl.h>
 
 #include <algorithm>
 #include <cstring>
+#include <vector>
 
 #include "internal.h"
 
@@ -225,6 +227,182 @@ isp_status_t isp_shard_exchange(isp_shard_ctx *ctx, void *strip, int elem_size, 
     if (s != ISP_OK) return s;
     if (cudaSetDevice(ctx->device) != cudaSuccess) return ispi_fail(ISP_ECUDA, "cudaSetDevice");
     return sc.n_ops > 0 ? post_exchange(ctx, sc, strip, (size_t)elem_size, pitch, (cudaStream_t)comm_stream) : ISP_OK;
+}
+
+}  // extern "C"
+
+// ---------------------------------------------------------------------------------
+// Peer-direct strips: no halo rows, no exchange.  Each rank's strip
+// holds only its own rows; the launch reads the hy rows above / below straight from the
+// neighbours' strips (peer memory over NVLink: CUDA IPC across processes, or any pointer
+// the device can dereference), so one launch covers the whole strip and nothing waits for
+// communication.  The strip-edge block rows are T / B regions that select the neighbour
+// buffer per row (row_base in isp_core.cuh); Body rows never leave the strip.
+// ---------------------------------------------------------------------------------
+namespace {
+
+template <class T>
+isp_status_t peer_rowrange(const T *own, const T *prev, const T *next, int H, int pitch, int rank, int nranks,
+                           int hy, int mode, RowRange &rr, const T *&base)
+{
+    int y0, sh;
+    isp_status_t s = isp_shard_rows(H, rank, nranks, &y0, &sh);
+    if (s != ISP_OK) return s;
+    const bool ring = mode == ISP_REPEAT && nranks > 1;
+    const int pr = rank > 0 ? rank - 1 : (ring ? nranks - 1 : -1);
+    const int nx = rank < nranks - 1 ? rank + 1 : (ring ? 0 : -1);
+    for (int r : {pr, nx}) {
+        if (r < 0) continue;
+        int a, b;
+        isp_shard_rows(H, r, nranks, &a, &b);
+        if (b < hy) return ispi_fail(ISP_EINVAL, "peer strip of rank %d has %d rows < hy = %d", r, b, hy);
+    }
+    if ((pr >= 0 && !prev) || (nx >= 0 && !next)) return ispi_fail(ISP_EINVAL, "missing neighbour strip pointer");
+    rr = RowRange{y0, sh, y0 + sh + hy, pr < 0, nx < 0};
+    rr.peer = 1;
+    rr.own_y0 = y0;
+    rr.own_y1 = y0 + sh;
+    base = own - (ptrdiff_t)y0 * pitch;
+    if (pr >= 0) {   // rows y < y0 of rank pr (rank 0 in a ring: global rows y + H)
+        int py0, psh;
+        isp_shard_rows(H, pr, nranks, &py0, &psh);
+        rr.peer_lo = prev - ((ptrdiff_t)py0 - (rank == 0 ? H : 0)) * pitch;
+    }
+    if (nx >= 0) {   // rows y >= y0 + sh of rank nx (last rank in a ring: global rows y - H)
+        int ny0, nsh;
+        isp_shard_rows(H, nx, nranks, &ny0, &nsh);
+        rr.peer_hi = next - ((ptrdiff_t)ny0 + (rank == nranks - 1 ? H : 0)) * pitch;
+    }
+    return ISP_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+isp_status_t isp_shard_filter_peer_local_f32(const float *own, const float *prev, const float *next, int w, int H,
+                                             int pitch, int rank, int nranks, const float *mask, int mw, int mh,
+                                             int border_mode, float const_val, float *out, int out_pitch,
+                                             isp_variant_t variant, isp_stream_t stream)
+{
+    if (!own || !out || !mask) return ispi_fail(ISP_EINVAL, "null pointer");
+    if (border_mode < 0 || border_mode > 3) return ispi_fail(ISP_EINVAL, "border mode %d", border_mode);
+    RowRange rr{};
+    const float *base = nullptr;
+    isp_status_t s = peer_rowrange(own, prev, next, H, pitch, rank, nranks, mh / 2, border_mode, rr, base);
+    if (s != ISP_OK) return s;
+    return ispi_filter_f32(base, w, H, pitch, mask, mw, mh, border_mode, const_val, out, out_pitch, variant, stream,
+                           &rr);
+}
+
+isp_status_t isp_shard_filter_peer_local_u8(const uint8_t *own, const uint8_t *prev, const uint8_t *next, int w,
+                                            int H, int pitch, int rank, int nranks, const int32_t *mask, int mw,
+                                            int mh, int32_t divisor, int border_mode, int const_val, uint8_t *out,
+                                            int out_pitch, isp_variant_t variant, isp_stream_t stream)
+{
+    if (!own || !out || !mask) return ispi_fail(ISP_EINVAL, "null pointer");
+    if (border_mode < 0 || border_mode > 3) return ispi_fail(ISP_EINVAL, "border mode %d", border_mode);
+    RowRange rr{};
+    const uint8_t *base = nullptr;
+    isp_status_t s = peer_rowrange(own, prev, next, H, pitch, rank, nranks, mh / 2, border_mode, rr, base);
+    if (s != ISP_OK) return s;
+    return ispi_filter_u8(base, w, H, pitch, mask, mw, mh, divisor, border_mode, const_val, out, out_pitch, variant,
+                          stream, &rr);
+}
+
+}  // extern "C"
+
+struct isp_shard_peer {
+    isp_shard_ctx *ctx;
+    void *own;
+    void *prev, *next;        // neighbour strips (opened IPC mappings), or null
+    void *prev_base, *next_base;
+};
+
+namespace {
+struct PeerInfo {
+    cudaIpcMemHandle_t h;
+    unsigned long long off;
+};
+}  // namespace
+
+extern "C" {
+
+isp_status_t isp_shard_peer_open(isp_shard_ctx *ctx, void *strip, int ring, isp_shard_peer **out)
+{
+    if (!ctx || !strip || !out) return ispi_fail(ISP_EINVAL, "isp_shard_peer_open args");
+    if (cudaSetDevice(ctx->device) != cudaSuccess) return ispi_fail(ISP_ECUDA, "cudaSetDevice");
+    // allocation base of the strip (IPC handles name allocations; torch's caching
+    // allocator hands out sub-ranges): cuMemGetAddressRange through the runtime's driver
+    // entry point, so libisp.so does not link libcuda (CPU boxes load it without a driver)
+    using AddrRangeFn = CUresult (*)(CUdeviceptr *, size_t *, CUdeviceptr);
+    void *fnp = nullptr;
+    cudaDriverEntryPointQueryResult q{};
+    if (cudaGetDriverEntryPoint("cuMemGetAddressRange", &fnp, cudaEnableDefault, &q) != cudaSuccess || !fnp)
+        return ispi_fail(ISP_ECUDA, "cuMemGetAddressRange entry point unavailable");
+    CUdeviceptr base = 0;
+    size_t size = 0;
+    if (((AddrRangeFn)fnp)(&base, &size, (CUdeviceptr)strip) != CUDA_SUCCESS)
+        return ispi_fail(ISP_ECUDA, "cuMemGetAddressRange of the strip failed");
+    PeerInfo mine{};
+    cudaError_t e = cudaIpcGetMemHandle(&mine.h, (void *)base);
+    if (e != cudaSuccess) return ispi_fail(ISP_ECUDA, "cudaIpcGetMemHandle: %s", cudaGetErrorString(e));
+    mine.off = (unsigned long long)((CUdeviceptr)strip - base);
+    const int P = ctx->nranks;
+    PeerInfo *dsend = nullptr, *drecv = nullptr;
+    std::vector<PeerInfo> all(P);
+    cudaStream_t st;
+    if (cudaMalloc(&dsend, sizeof(PeerInfo)) != cudaSuccess || cudaMalloc(&drecv, sizeof(PeerInfo) * P) != cudaSuccess ||
+        cudaStreamCreate(&st) != cudaSuccess)
+        return ispi_fail(ISP_ECUDA, "peer handle exchange buffers");
+    cudaMemcpy(dsend, &mine, sizeof(PeerInfo), cudaMemcpyHostToDevice);
+    isp_status_t s = nccl_status(ncclAllGather(dsend, drecv, sizeof(PeerInfo), ncclUint8, ctx->comm, st),
+                                 "ncclAllGather(ipc handles)");
+    if (s == ISP_OK && cudaStreamSynchronize(st) != cudaSuccess) s = ispi_fail(ISP_ECUDA, "handle exchange");
+    if (s == ISP_OK) cudaMemcpy(all.data(), drecv, sizeof(PeerInfo) * P, cudaMemcpyDeviceToHost);
+    cudaFree(dsend);
+    cudaFree(drecv);
+    cudaStreamDestroy(st);
+    if (s != ISP_OK) return s;
+    isp_shard_peer *pp = new isp_shard_peer{};
+    pp->ctx = ctx;
+    pp->own = strip;
+    const int r = ctx->rank;
+    const int pr = r > 0 ? r - 1 : ((ring && P > 1) ? P - 1 : -1);
+    const int nx = r < P - 1 ? r + 1 : ((ring && P > 1) ? 0 : -1);
+    auto open = [&](int q, void *&basep, void *&ptr) -> isp_status_t {
+        if (q < 0 || q == r) return ISP_OK;
+        cudaError_t ee = cudaIpcOpenMemHandle(&basep, all[q].h, cudaIpcMemLazyEnablePeerAccess);
+        if (ee != cudaSuccess) return ispi_fail(ISP_ECUDA, "cudaIpcOpenMemHandle(rank %d): %s", q, cudaGetErrorString(ee));
+        ptr = (char *)basep + all[q].off;
+        return ISP_OK;
+    };
+    if ((s = open(pr, pp->prev_base, pp->prev)) != ISP_OK || (s = open(nx, pp->next_base, pp->next)) != ISP_OK) {
+        isp_shard_peer_close(pp);
+        return s;
+    }
+    *out = pp;
+    return ISP_OK;
+}
+
+isp_status_t isp_shard_peer_filter_f32(isp_shard_peer *pp, int w, int H, int pitch, const float *mask, int mw, int mh,
+                                       int border_mode, float const_val, float *out, int out_pitch,
+                                       isp_variant_t variant, isp_stream_t stream)
+{
+    if (!pp) return ispi_fail(ISP_EINVAL, "null peer context");
+    if (cudaSetDevice(pp->ctx->device) != cudaSuccess) return ispi_fail(ISP_ECUDA, "cudaSetDevice");
+    return isp_shard_filter_peer_local_f32((const float *)pp->own, (const float *)pp->prev, (const float *)pp->next, w,
+                                           H, pitch, pp->ctx->rank, pp->ctx->nranks, mask, mw, mh, border_mode,
+                                           const_val, out, out_pitch, variant, stream);
+}
+
+isp_status_t isp_shard_peer_close(isp_shard_peer *pp)
+{
+    if (!pp) return ISP_OK;
+    if (pp->prev_base) cudaIpcCloseMemHandle(pp->prev_base);
+    if (pp->next_base && pp->next_base != pp->prev_base) cudaIpcCloseMemHandle(pp->next_base);
+    delete pp;
+    return ISP_OK;
 }
 
 isp_status_t isp_shard_destroy(isp_shard_ctx *ctx)

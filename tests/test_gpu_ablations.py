@@ -92,10 +92,11 @@ def test_split_other_ops(isp):
 
 
 @pytest.mark.parametrize("name", list(MASKS))
-@pytest.mark.parametrize("shape", [(70, 2052), (45, 333), (5, 7)])
+@pytest.mark.parametrize("shape", [(70, 2048), (45, 328), (5, 8)])
 def test_tex_f32(isp, name, shape):
     """Texture address modes reproduce the four patterns, windows larger than the image
-    included (5x7 image, 9x9 window: wrap / mirror periods handled by the hardware)."""
+    included (5x8 image, 9x9 window: wrap / mirror periods handled by the hardware).
+    Widths keep rows on the device's texture pitch alignment (32 B)."""
     mask = MASKS[name]
     h, w = shape
     img = synth.uniform_f32(h, w, 74)
@@ -104,6 +105,12 @@ def test_tex_f32(isp, name, shape):
         ref, sc = oracle.filter_f64(img, mask, mode, 0.25, with_scale=True)
         got = host(isp.isp_filter_ex(d, mask, mode, 0.25, variant="tex"))
         check_f32(got, ref, sc)
+
+
+def test_tex_needs_pitch_alignment(isp):
+    img = dev(synth.uniform_f32(16, 2052, 1))        # 8208-B rows: not a multiple of 32 B
+    with pytest.raises(isp.IspError):
+        isp.isp_filter_ex(img, MASKS["rand5"], "clamp", 0.0, variant="tex")
 
 
 def test_tex_unsupported_elsewhere(isp):

@@ -421,3 +421,57 @@ def test_sobel_magnitude_near_ties(isp):
             dx, dy, mag = isp.isp_sobel_u8(d, mode, 0, variant=v)
             ran(isp, v)
             np.testing.assert_array_equal(host(mag), rmag, err_msg=f"{mode} {v}")
+
+
+# ---------------------------------------------------------------- peer-direct strips (N4)
+@pytest.mark.parametrize("nranks", [2, 3, 8])
+@pytest.mark.parametrize("m", [3, 7, 9])
+def test_peer_strips_f32(isp, nranks, m):
+    """Peer-direct strips: every rank's buffer holds only its own rows,
+    the neighbour rows are read from the neighbours' buffers (separate allocations, as
+    IPC mappings would be), ONE launch per rank; the gathered result equals the
+    single-image result bitwise, strip-edge block rows run T / B bodies (non-degenerate)."""
+    H, W = 203, 2052
+    img = synth.uniform_f32(H, W, 79)
+    mask = np.random.default_rng(m).random((m, m)).astype(np.float32)
+    full = dev(img)
+    strips = []
+    for r in range(nranks):
+        y0, sh = isp.isp_shard_rows(H, r, nranks)
+        strips.append(dev(img[y0:y0 + sh]))
+    for mode in MODES:
+        ring = mode == "repeat"
+        for v in ["tma", "warp", "naive"]:
+            ref = host(isp.isp_filter_ex(full, mask, mode, 0.25, variant=v))
+            got = np.full((H, W), np.nan, dtype=np.float32)
+            for r in range(nranks):
+                y0, sh = isp.isp_shard_rows(H, r, nranks)
+                prev = strips[r - 1] if r > 0 else (strips[-1] if ring else None)
+                nxt = strips[r + 1] if r < nranks - 1 else (strips[0] if ring else None)
+                isp.isp_clear_plans()
+                out = isp.isp_shard_filter_peer_local_f32(strips[r], prev, nxt, H, r, nranks, mask, mode, 0.25,
+                                                          variant=v)
+                plans = isp.isp_recent_plans()
+                assert len(plans) == 1 and not plans[0]["degenerate"], plans
+                got[y0:y0 + sh] = host(out)
+            np.testing.assert_array_equal(got, ref, err_msg=f"{mode} {v} P={nranks} m={m}")
+
+
+@pytest.mark.parametrize("nranks", [2, 4])
+def test_peer_strips_u8(isp, nranks):
+    H, W = 150, 2064
+    img = synth.uniform_u8(H, W, 80)
+    mask, div = oracle.gaussian_u8_mask(5)
+    strips = [dev(img[slice(*(lambda y, s: (y, y + s))(*isp.isp_shard_rows(H, r, nranks)))]) for r in range(nranks)]
+    for mode in MODES:
+        ring = mode == "repeat"
+        ref = oracle.filter_u8(img, mask, div, mode, 9)
+        for v in ["warp", "tma", "naive"]:
+            got = np.zeros((H, W), dtype=np.uint8)
+            for r in range(nranks):
+                y0, sh = isp.isp_shard_rows(H, r, nranks)
+                prev = strips[r - 1] if r > 0 else (strips[-1] if ring else None)
+                nxt = strips[r + 1] if r < nranks - 1 else (strips[0] if ring else None)
+                got[y0:y0 + sh] = host(isp.isp_shard_filter_peer_local_u8(strips[r], prev, nxt, H, r, nranks, mask,
+                                                                          div, mode, 9, variant=v))
+            np.testing.assert_array_equal(got, ref, err_msg=f"{mode} {v} P={nranks}")

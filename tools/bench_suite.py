@@ -46,7 +46,7 @@ def time_launch(fn, nbuf, R=12, reps=20):
     """fn(i) launches one kernel on buffer set i % nbuf on the current stream."""
     stream = torch.cuda.Stream()
     with torch.cuda.stream(stream):
-        for i in range(2):
+        for i in range(max(2, min(nbuf, R))):   # every buffer once: per-buffer host state (texture objects) exists before capture
             fn(i)
     torch.cuda.synchronize()
     plan = isp.isp_last_plan()
