@@ -21,6 +21,8 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <algorithm>
+#include <cstdlib>
 #include <cstring>
 
 #include "../../include/isp.h"
@@ -109,7 +111,10 @@ struct Params {
     long long thr;
     int16_t *dx, *dy;
     uint8_t *mag, *lap, *har;
+    // tile-ISP kernel (round 2): tiles [bx0, bx1) x [by0, by1) are its Body region
+    int nbx, nby, bx0, bx1, by0, by1;
 };
+
 
 __global__ void __launch_bounds__(NT, FUSED_MINB) k_fused_cfg3(const Params p)
 {
@@ -286,6 +291,366 @@ __global__ void __launch_bounds__(NT, FUSED_MINB) k_fused_cfg3(const Params p)
     (void)cx0; (void)cy0;
 }
 
+// =====================================================================================
+// Body-tile kernel (round 2).  Runs only tiles whose whole staged window lies inside the
+// image (the Body region of the tile partition, Listing 3 at tile granularity): no checks,
+// no remapped ext positions, so it can be built for instruction count and occupancy:
+//   * Sobel's horizontal parts on 16-bit pair lanes (SWAR: pixels (0,2) and (1,3) of a
+//     4-pixel group share one 32-bit register; all lanes stay in [0, 65535], biased where
+//     a value can be negative, so no carry / borrow crosses lanes);
+//   * the dx / dy ext grid in shared memory as exact floats (|dx|, |dy| <= 1020);
+//   * Harris window sums with packed FP32x2 FMAs (exact: integers < 2^24), the response
+//     in f32 with a rigorous error bound and the exact f64 evaluation only when the bound
+//     cannot decide R25 > thr;
+//   * Laplace horizontal 5-sums with DP4A on byte windows, vertical sums in a 5-row ring.
+// Output bits equal the general kernel's (and the oracle composition's).
+// =====================================================================================
+constexpr int G2 = 34;                                  // ext groups: cols x0-4+4G .. x0-1+4G
+constexpr int EWF = 4 * G2;                             // floats per ext row
+constexpr int NSEG2 = NT / G2, SEGR2 = (EH + NSEG2 - 1) / NSEG2;
+#ifndef FUSED_BODY_MINB
+#define FUSED_BODY_MINB 5
+#endif
+
+struct BodySmem {
+    uint8_t in[SH][SW];                                 // image rows y0-2.., cols x0-16..
+    float fx[EH][EWF], fy[EH][EWF];                     // per group [p0, p2, p1, p3]
+};
+
+__device__ __forceinline__ uint32_t lw(const uint8_t *p) { return *reinterpret_cast<const uint32_t *>(p); }
+
+// 16-bit lanes (biased by 1024) -> exact floats: 2^23 + lane has the lane in its mantissa
+__device__ __forceinline__ float2 lanes_f(uint32_t x)
+{
+    const float b = 8388608.0f + 1024.0f;
+    return make_float2(__uint_as_float(__byte_perm(x, 0x4B000000u, 0x7610)) - b,
+                       __uint_as_float(__byte_perm(x, 0x4B000000u, 0x7632)) - b);
+}
+
+// Sobel horizontal parts of one staged row for the 4 pixels at s_in column c (pairs:
+// E = pixels (0, 2), O = (1, 3)): s = a + 2b + c, d = c - a + 256 (bias).
+__device__ __forceinline__ void hsob(const uint8_t *row, int c, uint32_t &sE, uint32_t &sO, uint32_t &dE,
+                                     uint32_t &dO)
+{
+    const uint32_t A = lw(row + c - 4), B = lw(row + c), C = lw(row + c + 4);
+    const uint32_t Ec = __byte_perm(B, 0u, 0x4240), Oc = __byte_perm(B, 0u, 0x4341);
+    const uint32_t El = __byte_perm(A, B, 0x0503) & 0x00FF00FFu;   // (c-1, c1)
+    const uint32_t Or = __byte_perm(B, C, 0x0402) & 0x00FF00FFu;   // (c2, c4)
+    sE = El + 2u * Ec + Oc;
+    sO = Ec + 2u * Oc + Or;
+    dE = Oc + 0x01000100u - El;
+    dO = Or + 0x01000100u - Ec;
+}
+
+__device__ __forceinline__ float2 f2(float a, float b) { return make_float2(a, b); }
+__device__ __forceinline__ float2 mul2(float2 a, float2 b)
+{
+    unsigned long long x, y, z;
+    asm("mov.b64 %0, {%1, %2};" : "=l"(x) : "f"(a.x), "f"(a.y));
+    asm("mov.b64 %0, {%1, %2};" : "=l"(y) : "f"(b.x), "f"(b.y));
+    asm("mul.rn.f32x2 %0, %1, %2;" : "=l"(z) : "l"(x), "l"(y));
+    float2 r;
+    asm("mov.b64 {%0, %1}, %2;" : "=f"(r.x), "=f"(r.y) : "l"(z));
+    return r;
+}
+__device__ __forceinline__ float2 fma2(float2 a, float2 b, float2 c)
+{
+    unsigned long long x, y, z, w;
+    asm("mov.b64 %0, {%1, %2};" : "=l"(x) : "f"(a.x), "f"(a.y));
+    asm("mov.b64 %0, {%1, %2};" : "=l"(y) : "f"(b.x), "f"(b.y));
+    asm("mov.b64 %0, {%1, %2};" : "=l"(z) : "f"(c.x), "f"(c.y));
+    asm("fma.rn.f32x2 %0, %1, %2, %3;" : "=l"(w) : "l"(x), "l"(y), "l"(z));
+    float2 r;
+    asm("mov.b64 {%0, %1}, %2;" : "=f"(r.x), "=f"(r.y) : "l"(w));
+    return r;
+}
+__device__ __forceinline__ float2 add2(float2 a, float2 b)
+{
+    unsigned long long x, y, z;
+    asm("mov.b64 %0, {%1, %2};" : "=l"(x) : "f"(a.x), "f"(a.y));
+    asm("mov.b64 %0, {%1, %2};" : "=l"(y) : "f"(b.x), "f"(b.y));
+    asm("add.rn.f32x2 %0, %1, %2;" : "=l"(z) : "l"(x), "l"(y));
+    float2 r;
+    asm("mov.b64 {%0, %1}, %2;" : "=f"(r.x), "=f"(r.y) : "l"(z));
+    return r;
+}
+
+// Horizontal [1,2,1] sums of xx, yy, xy over ext row e for the 4 pixels of group G, as
+// pairs (H(p0), H(p2)) and (H(p1), H(p3)).  Exact: integer products / sums < 2^24.
+struct HS { float2 xxE, xxO, yyE, yyO, xyE, xyO; };
+__device__ __forceinline__ HS hsum_row(const float *fxr, const float *fyr, int G)
+{
+    const float4 X = *reinterpret_cast<const float4 *>(fxr + 4 * G);     // p0, p2, p1, p3
+    const float4 Y = *reinterpret_cast<const float4 *>(fyr + 4 * G);
+    const float xl = fxr[4 * G - 1], yl = fyr[4 * G - 1];                 // p-1 (left group's p3)
+    const float xr = fxr[4 * G + 4], yr = fyr[4 * G + 4];                 // p4 (right group's p0)
+    const float2 xE = f2(X.x, X.y), xO = f2(X.z, X.w), yE = f2(Y.x, Y.y), yO = f2(Y.z, Y.w);
+    // products at positions: E = (p0, p2), O = (p1, p3), A = (p-1, p1), B = (p2, p4)
+    const float2 xxE = mul2(xE, xE), xxO = mul2(xO, xO), yyE = mul2(yE, yE), yyO = mul2(yO, yO);
+    const float2 xyE = mul2(xE, yE), xyO = mul2(xO, yO);
+    const float2 xxA = f2(xl * xl, xxO.x), xxB = f2(xxE.y, xr * xr);
+    const float2 yyA = f2(yl * yl, yyO.x), yyB = f2(yyE.y, yr * yr);
+    const float2 xyA = f2(xl * yl, xyO.x), xyB = f2(xyE.y, xr * yr);
+    const float2 two = f2(2.f, 2.f);
+    HS h;
+    h.xxE = add2(fma2(two, xxE, xxA), xxO);   // (H0, H2) = A + 2E + O
+    h.xxO = add2(fma2(two, xxO, xxE), xxB);   // (H1, H3) = E + 2O + B
+    h.yyE = add2(fma2(two, yyE, yyA), yyO);
+    h.yyO = add2(fma2(two, yyO, yyE), yyB);
+    h.xyE = add2(fma2(two, xyE, xyA), xyO);
+    h.xyO = add2(fma2(two, xyO, xyE), xyB);
+    return h;
+}
+
+// R25 > thr for a pair of pixels from exact window sums (floats, integers < 2^24).
+// Fast f32 path: |R_f - R| <= 2^-17 (p + q + t^2) (generous bound on five roundings,
+// DESIGN.md 7g); undecided pixels take the exact f64 evaluation of the general kernel.
+__device__ __forceinline__ void harris2(float2 sxx, float2 syy, float2 sxy, float thr_f, float thr_err, double thr,
+                                        int &o0, int &o1)
+{
+    const float2 p = mul2(sxx, syy), q = mul2(sxy, sxy);
+    const float2 det = fma2(f2(-sxy.x, -sxy.y), sxy, p);
+    const float2 t = add2(sxx, syy);
+    const float2 tt = mul2(t, t);
+    const float2 R = fma2(f2(25.f, 25.f), det, f2(-tt.x, -tt.y));
+    const float2 bnd = add2(add2(p, q), tt);
+    const float b0 = fmaf(bnd.x, 7.62939453125e-06f, thr_err), b1 = fmaf(bnd.y, 7.62939453125e-06f, thr_err);
+    const float d0 = R.x - thr_f, d1 = R.y - thr_f;
+    o0 = d0 > b0 ? 255 : 0;
+    o1 = d1 > b1 ? 255 : 0;
+    // undecided: all window sums zero (flat image area) -> R25 = 0 exactly; otherwise the
+    // exact f64 evaluation (rare)
+    const int zero_dec = 0.0 > thr ? 255 : 0;
+    if (!(d0 > b0 || -d0 > b0)) {
+        if (bnd.x == 0.f) {
+            o0 = zero_dec;
+        } else {
+            const double dx = sxx.x, dy = syy.x, dz = sxy.x;
+            const double dd = fma(-dz, dz, dx * dy), tr = dx + dy;
+            o0 = fma(25.0, dd, -(tr * tr)) > thr ? 255 : 0;
+        }
+    }
+    if (!(d1 > b1 || -d1 > b1)) {
+        if (bnd.y == 0.f) {
+            o1 = zero_dec;
+        } else {
+            const double dx = sxx.y, dy = syy.y, dz = sxy.y;
+            const double dd = fma(-dz, dz, dx * dy), tr = dx + dy;
+            o1 = fma(25.0, dd, -(tr * tr)) > thr ? 255 : 0;
+        }
+    }
+}
+
+__device__ __forceinline__ int mag_f(float n)
+{
+    float r;
+    asm("sqrt.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(fminf(n, 65280.0f)));
+    return (int)(r + 0.5f);
+}
+
+// Border tile staging: rows through the pattern once per row; 16-byte vectors whose columns
+// are all inside the image are copied as vectors, the rest byte by byte through the pattern
+// (the Body-tile launch requires w, h >= 2 tiles, so overshoots stay below N).
+__device__ __noinline__ void stage_border(const Params &p, uint8_t *in, int x0, int y0)
+{
+    constexpr int VPR = SW / 16;
+    for (int k = threadIdx.x; k < SH * VPR; k += NT) {
+        const int r = k / VPR, c = k % VPR;
+        const int yy = bmap(p.mode, y0 - 2 + r, p.h);          // -1: Constant, row outside
+        uint8_t *dst = in + r * SW + 16 * c;
+        const int xs = x0 - XO + 16 * c;
+        if (yy >= 0 && xs >= 0 && xs + 16 <= p.w) {
+            *reinterpret_cast<uint4 *>(dst) = __ldg(reinterpret_cast<const uint4 *>(p.img + (size_t)yy * p.pitch + xs));
+        } else {
+            for (int e = 0; e < 16; ++e) {
+                const int xx = bmap(p.mode, xs + e, p.w);
+                dst[e] = (uint8_t)((yy < 0 || xx < 0) ? p.cval : p.img[(size_t)yy * p.pitch + xx]);
+            }
+        }
+    }
+}
+
+// Ext grid positions the stored outputs read that lie outside the image (x = -1 or w,
+// y = -1 or h): the Sobel value of the remapped pixel (or the Harris constant).
+__device__ __forceinline__ int ext_slot(int gx, int x0)   // ext column slot of image column gx
+{
+    const int rel = gx - (x0 - 4), G = rel >> 2, pos = rel & 3;   // slots hold p0, p2, p1, p3
+    return 4 * G + (pos == 0 ? 0 : pos == 1 ? 2 : pos == 2 ? 1 : 3);
+}
+
+__device__ __noinline__ void fix_ext_border(const Params &p, float *fx, float *fy, int x0, int y0)
+{
+    const int w = p.w, h = p.h;
+    auto fix = [&](int gx, int gy) {
+        int16_t vx, vy;
+        fix_ext(p, gx, gy, &vx, &vy);
+        const int k = (gy - (y0 - 1)) * EWF + ext_slot(gx, x0);
+        fx[k] = (float)vx;
+        fy[k] = (float)vy;
+    };
+    // columns x = -1 and x = w (rows y in [-1, h])
+    for (int k = threadIdx.x; k < 2 * EH; k += NT) {
+        const int gy = y0 - 1 + (k >> 1), gx = (k & 1) ? w : -1;
+        if (gx >= x0 - 4 && gx < x0 - 4 + EWF && gy >= -1 && gy <= h) fix(gx, gy);
+    }
+    // rows y = -1 and y = h (columns inside the image; the corners were done above)
+    for (int k = threadIdx.x; k < 2 * EWF; k += NT) {
+        const int gy = k < EWF ? -1 : h, gx = x0 - 4 + (k % EWF);
+        if (gy >= y0 - 1 && gy < y0 - 1 + EH && gx >= 0 && gx < w) fix(gx, gy);
+    }
+}
+
+// Tile order of the tile-ISP launch: the border tiles (slow: patterned staging, ext fix-ups)
+// first, so they do not trail the last wave; then the Body tiles row-major.
+__device__ __forceinline__ void tile_of(const Params &p, int k, int &bx, int &by)
+{
+    const int nb_in = (p.bx1 - p.bx0) * (p.by1 - p.by0), nframe = p.nbx * p.nby - nb_in;
+    if (k >= nframe) {
+        k -= nframe;
+        const int iw = p.bx1 - p.bx0;
+        bx = p.bx0 + k % iw;
+        by = p.by0 + k / iw;
+        return;
+    }
+    const int inner_w = p.bx1 - p.bx0, per_mid = p.nbx - inner_w;
+    const int top = p.by0 * p.nbx, mid = (p.by1 - p.by0) * per_mid;
+    if (k < top) { by = k / p.nbx; bx = k % p.nbx; return; }
+    k -= top;
+    if (k < mid) {
+        by = p.by0 + k / per_mid;
+        const int j = k % per_mid;
+        bx = j < p.bx0 ? j : j + inner_w;
+        return;
+    }
+    k -= mid;
+    by = p.by1 + k / p.nbx;
+    bx = k % p.nbx;
+}
+
+__global__ void __launch_bounds__(NT, FUSED_BODY_MINB) k_fused_body(const Params p)
+{
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    BodySmem &S = *reinterpret_cast<BodySmem *>(smem_raw);
+    const int tid = threadIdx.x;
+    int bx, by;
+    tile_of(p, (int)blockIdx.x, bx, by);
+    const int x0 = bx * TW, y0 = by * TH;
+    // Listing 3 at tile granularity: Body tiles read their whole window unchecked; border
+    // tiles stage through the border pattern and fix up the ext positions outside the image
+    const bool body = bx >= p.bx0 && bx < p.bx1 && by >= p.by0 && by < p.by1;
+
+    // ---- stage img rows y0-2 .. y0+TH+1, cols x0-16 .. x0+TW+15 -------------------------
+    if (body) {
+        constexpr int VPR = SW / 16;
+        for (int k = tid; k < SH * VPR; k += NT) {
+            const int r = k / VPR, c = k % VPR;
+            const uint4 v = __ldg(reinterpret_cast<const uint4 *>(p.img + (size_t)(y0 - 2 + r) * p.pitch + x0 - XO) + c);
+            *reinterpret_cast<uint4 *>(&S.in[r][c * 16]) = v;
+        }
+    } else {
+        stage_border(p, &S.in[0][0], x0, y0);
+    }
+    __syncthreads();
+
+    // ---- dx, dy on the ext grid (rows y0-1 .. y0+TH, cols x0-4 .. x0+TW+3) -------------
+    for (int it = tid; it < G2 * NSEG2; it += NT) {
+        const int G = it % G2, rs = (it / G2) * SEGR2, re = min(EH, rs + SEGR2);
+        const int c = 12 + 4 * G;                           // s_in column of the group
+        uint32_t sE0, sO0, dE0, dO0, sE1, sO1, dE1, dO1;
+        hsob(S.in[rs], c, sE0, sO0, dE0, dO0);
+        hsob(S.in[rs + 1], c, sE1, sO1, dE1, dO1);
+        for (int er = rs; er < re; ++er) {
+            uint32_t sE2, sO2, dE2, dO2;
+            hsob(S.in[er + 2], c, sE2, sO2, dE2, dO2);
+            const uint32_t dxE = dE0 + 2u * dE1 + dE2, dxO = dO0 + 2u * dO1 + dO2;   // + 1024 per lane
+            const uint32_t dyE = sE2 + 0x04000400u - sE0, dyO = sO2 + 0x04000400u - sO0;
+            const float2 xE = lanes_f(dxE), xO = lanes_f(dxO), yE = lanes_f(dyE), yO = lanes_f(dyO);
+            *reinterpret_cast<float4 *>(&S.fx[er][4 * G]) = make_float4(xE.x, xE.y, xO.x, xO.y);
+            *reinterpret_cast<float4 *>(&S.fy[er][4 * G]) = make_float4(yE.x, yE.y, yO.x, yO.y);
+            sE0 = sE1; sO0 = sO1; dE0 = dE1; dO0 = dO1;
+            sE1 = sE2; sO1 = sO2; dE1 = dE2; dO1 = dO2;
+        }
+    }
+    if (!body) {   // ext positions outside the image: dx/dy of the remapped pixel (Harris' input)
+        __syncthreads();
+        fix_ext_border(p, &S.fx[0][0], &S.fy[0][0], x0, y0);
+    }
+    __syncthreads();
+
+    // ---- outputs: lane -> 4 columns (group G = lane + 1), warp -> RPW rows ----------------
+    const int lane = tid & 31, G = lane + 1;
+    const int xr = 4 * lane, x = x0 + xr;
+    const int rbeg = (tid >> 5) * RPW, rend = min(rbeg + RPW, p.h - y0);
+    if (rbeg >= rend || x >= p.w) return;   // rows / columns past the image (partial tiles)
+    const bool full = body || (x + 3 < p.w);
+    const double thr = (double)max(-9007199254740992ll, min(9007199254740992ll, p.thr));
+    const float thr_f = (float)thr;
+    const float thr_err = 2.0f * 5.9604645e-08f * fabsf(thr_f) + 1e-30f;    // |(float)thr - thr| + margin
+    const uint32_t ones = 0x01010101u;
+    // Laplace: horizontal 5-sums of staged row sr at the 4 pixels (DP4A on byte windows)
+    auto h5 = [&](int sr, int (&H)[4]) {
+        const uint8_t *row = S.in[sr] + XO + xr;
+        const uint32_t L = lw(row - 4), B = lw(row), R = lw(row + 4);
+        H[0] = (int)__dp4a(__funnelshift_r(L, B, 16), ones, (B >> 16) & 0xffu);
+        H[1] = (int)__dp4a(__funnelshift_r(L, B, 24), ones, B >> 24);
+        H[2] = (int)__dp4a(B, ones, R & 0xffu);
+        H[3] = (int)__dp4a(__funnelshift_r(B, R, 8), ones, (R >> 8) & 0xffu);
+    };
+    int H0[4], H1[4], H2[4], H3[4];
+    h5(rbeg, H0); h5(rbeg + 1, H1); h5(rbeg + 2, H2); h5(rbeg + 3, H3);
+    HS a = hsum_row(S.fx[rbeg], S.fy[rbeg], G), b = hsum_row(S.fx[rbeg + 1], S.fy[rbeg + 1], G);
+#pragma unroll 1
+    for (int r = rbeg; r < rend; ++r) {
+        const size_t off = (size_t)(y0 + r) * p.out_pitch + x;
+        // Laplace (a8): box - 25 centre, clamped
+        int H4[4];
+        h5(r + 4, H4);
+        const uint32_t cw = lw(S.in[r + 2] + XO + xr);
+        uint32_t lapw = 0;
+#pragma unroll
+        for (int k = 0; k < 4; ++k) {
+            const int v = H0[k] + H1[k] + H2[k] + H3[k] + H4[k] - 25 * (int)((cw >> (8 * k)) & 0xff);
+            lapw |= (uint32_t)min(255, max(0, v)) << (8 * k);
+            H0[k] = H1[k]; H1[k] = H2[k]; H2[k] = H3[k]; H3[k] = H4[k];
+        }
+        // Harris (a10) on ext rows r, r+1, r+2 (image rows y-1, y, y+1)
+        const HS c = hsum_row(S.fx[r + 2], S.fy[r + 2], G);
+        const float2 two = f2(2.f, 2.f);
+        const float2 sxxE = add2(fma2(two, b.xxE, a.xxE), c.xxE), sxxO = add2(fma2(two, b.xxO, a.xxO), c.xxO);
+        const float2 syyE = add2(fma2(two, b.yyE, a.yyE), c.yyE), syyO = add2(fma2(two, b.yyO, a.yyO), c.yyO);
+        const float2 sxyE = add2(fma2(two, b.xyE, a.xyE), c.xyE), sxyO = add2(fma2(two, b.xyO, a.xyO), c.xyO);
+        int h0, h1, h2, h3;
+        harris2(sxxE, syyE, sxyE, thr_f, thr_err, thr, h0, h2);
+        harris2(sxxO, syyO, sxyO, thr_f, thr_err, thr, h1, h3);
+        // Sobel magnitude (a9) and the optional dx / dy images, ext row r + 1
+        const float4 X = *reinterpret_cast<const float4 *>(&S.fx[r + 1][4 * G]);
+        const float4 Y = *reinterpret_cast<const float4 *>(&S.fy[r + 1][4 * G]);
+        const float2 nE = fma2(f2(X.x, X.y), f2(X.x, X.y), mul2(f2(Y.x, Y.y), f2(Y.x, Y.y)));
+        const float2 nO = fma2(f2(X.z, X.w), f2(X.z, X.w), mul2(f2(Y.z, Y.w), f2(Y.z, Y.w)));
+        const uint32_t magw = (uint32_t)mag_f(nE.x) | (uint32_t)mag_f(nO.x) << 8 | (uint32_t)mag_f(nE.y) << 16 |
+                              (uint32_t)mag_f(nO.y) << 24;
+        const uint32_t harw = (uint32_t)h0 | (uint32_t)h1 << 8 | (uint32_t)h2 << 16 | (uint32_t)h3 << 24;
+        if (full) {
+            *reinterpret_cast<uint32_t *>(p.lap + off) = lapw;
+            *reinterpret_cast<uint32_t *>(p.har + off) = harw;
+            *reinterpret_cast<uint32_t *>(p.mag + off) = magw;
+            if (p.dx) *reinterpret_cast<uint2 *>(p.dx + off) = make_uint2(pack16((int)X.x, (int)X.z), pack16((int)X.y, (int)X.w));
+            if (p.dy) *reinterpret_cast<uint2 *>(p.dy + off) = make_uint2(pack16((int)Y.x, (int)Y.z), pack16((int)Y.y, (int)Y.w));
+        } else {   // the image's last, partial 4-pixel group
+            const int dxv[4] = {(int)X.x, (int)X.z, (int)X.y, (int)X.w}, dyv[4] = {(int)Y.x, (int)Y.z, (int)Y.y, (int)Y.w};
+            for (int k = 0; k < 4 && x + k < p.w; ++k) {
+                p.lap[off + k] = (uint8_t)(lapw >> (8 * k));
+                p.har[off + k] = (uint8_t)(harw >> (8 * k));
+                p.mag[off + k] = (uint8_t)(magw >> (8 * k));
+                if (p.dx) p.dx[off + k] = (int16_t)dxv[k];
+                if (p.dy) p.dy[off + k] = (int16_t)dyv[k];
+            }
+        }
+        a = b;
+        b = c;
+    }
+}
+
 // Cold paths kept out of line (instruction-cache footprint of the hot loop).
 // dx/dy of the dx/dy IMAGES at an ext position outside the image: the Sobel value at the
 // remapped pixel B(gx), B(gy); Constant: the Harris constant.
@@ -358,9 +723,32 @@ extern "C" isp_status_t isp_pipeline_cfg3_u8(const uint8_t *img, int w, int h, i
                 (uintptr_t)harris % 4 == 0 && (!dx || (uintptr_t)dx % 8 == 0) && (!dy || (uintptr_t)dy % 8 == 0);
     p.thr = thr;
     p.dx = dx; p.dy = dy; p.mag = mag; p.lap = lap; p.har = harris;
-    const dim3 grid((w + TW - 1) / TW, (h + TH - 1) / TH);
-    k_fused_cfg3<<<grid, NT, 0, (cudaStream_t)stream>>>(p);
-    const cudaError_t e = cudaGetLastError();
+    const int nbx = (w + TW - 1) / TW, nby = (h + TH - 1) / TH;
+    p.nbx = nbx;
+    p.nby = nby;
+    // Body tiles (Listing 3 at tile granularity: the whole staged window inside the image,
+    // 16-B aligned rows, full 4-pixel stores): the fast Body kernel; the frame of border
+    // tiles: the general kernel.  ISP_NAIVE / unaligned images: the general kernel alone.
+    p.bx0 = 1;
+    p.bx1 = std::max(1, std::min(nbx, (w - TW - XO) / TW + 1));
+    p.by0 = 1;
+    p.by1 = std::max(1, std::min(nby, (h - TH - 2) / TH + 1));
+    // one launch of the tile-ISP kernel when the image is at least 2 x 2 tiles + halo (single
+    // reflections suffice at its borders); ISP_NAIVE, unaligned or tiny images: the general kernel
+    const bool body = !p.naive && p.vec && p.vec_out && p.bx1 > p.bx0 && p.by1 > p.by0 && w >= 2 * TW && h >= 2 * TH &&
+                      !getenv("ISP_FUSED_V1");
+    cudaError_t e = cudaSuccess;
+    if (body) {
+        static bool attr = false;
+        if (!attr) {
+            cudaFuncSetAttribute(k_fused_body, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(BodySmem));
+            attr = true;
+        }
+        k_fused_body<<<nbx * nby, NT, sizeof(BodySmem), (cudaStream_t)stream>>>(p);
+    } else {
+        k_fused_cfg3<<<dim3(nbx, nby), NT, 0, (cudaStream_t)stream>>>(p);
+    }
+    e = cudaGetLastError();
     if (e != cudaSuccess) return ispi_fail(ISP_ECUDA, "isp_pipeline_cfg3_u8: %s", cudaGetErrorString(e));
     return ISP_OK;
 }
