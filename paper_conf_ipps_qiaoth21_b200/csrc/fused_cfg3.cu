@@ -402,9 +402,18 @@ __device__ __forceinline__ HS hsum_row(const float *fxr, const float *fyr, int G
     return h;
 }
 
+// Exact R25 > thr (f64: every intermediate is an integer < 2^53).
+__device__ __noinline__ int harris_exact(float sxx, float syy, float sxy, double thr)
+{
+    const double dx = sxx, dy = syy, dz = sxy;
+    const double dd = fma(-dz, dz, dx * dy), tr = dx + dy;
+    return fma(25.0, dd, -(tr * tr)) > thr ? 255 : 0;
+}
+
 // R25 > thr for a pair of pixels from exact window sums (floats, integers < 2^24).
 // Fast f32 path: |R_f - R| <= 2^-17 (p + q + t^2) (generous bound on five roundings,
-// DESIGN.md 7g); undecided pixels take the exact f64 evaluation of the general kernel.
+// DESIGN.md 7g); a pixel the bound cannot decide takes the exact f64 evaluation (out of
+// line; all sums zero -- a flat area -- means R25 = 0 exactly).
 __device__ __forceinline__ void harris2(float2 sxx, float2 syy, float2 sxy, float thr_f, float thr_err, double thr,
                                         int &o0, int &o1)
 {
@@ -418,26 +427,10 @@ __device__ __forceinline__ void harris2(float2 sxx, float2 syy, float2 sxy, floa
     const float d0 = R.x - thr_f, d1 = R.y - thr_f;
     o0 = d0 > b0 ? 255 : 0;
     o1 = d1 > b1 ? 255 : 0;
-    // undecided: all window sums zero (flat image area) -> R25 = 0 exactly; otherwise the
-    // exact f64 evaluation (rare)
-    const int zero_dec = 0.0 > thr ? 255 : 0;
-    if (!(d0 > b0 || -d0 > b0)) {
-        if (bnd.x == 0.f) {
-            o0 = zero_dec;
-        } else {
-            const double dx = sxx.x, dy = syy.x, dz = sxy.x;
-            const double dd = fma(-dz, dz, dx * dy), tr = dx + dy;
-            o0 = fma(25.0, dd, -(tr * tr)) > thr ? 255 : 0;
-        }
-    }
-    if (!(d1 > b1 || -d1 > b1)) {
-        if (bnd.y == 0.f) {
-            o1 = zero_dec;
-        } else {
-            const double dx = sxx.y, dy = syy.y, dz = sxy.y;
-            const double dd = fma(-dz, dz, dx * dy), tr = dx + dy;
-            o1 = fma(25.0, dd, -(tr * tr)) > thr ? 255 : 0;
-        }
+    const bool u0 = fabsf(d0) <= b0, u1 = fabsf(d1) <= b1;     // undecided by the bound
+    if (__any_sync(0xffffffffu, u0 || u1)) {
+        if (u0) o0 = bnd.x == 0.f ? (0.0 > thr ? 255 : 0) : harris_exact(sxx.x, syy.x, sxy.x, thr);
+        if (u1) o1 = bnd.y == 0.f ? (0.0 > thr ? 255 : 0) : harris_exact(sxx.y, syy.y, sxy.y, thr);
     }
 }
 
@@ -448,6 +441,20 @@ __device__ __forceinline__ int mag_f(float n)
     return (int)(r + 0.5f);
 }
 
+// Border pattern for an overshoot below N (one reflection / wrap): the tile-ISP launch
+// only runs on images of at least 2 x 2 tiles, whose staged windows reach 16 columns and
+// 2 rows past the edge.
+__device__ __forceinline__ int bmap1(int mode, int i, int n)
+{
+    if (i >= 0 && i < n) return i;
+    switch (mode) {
+    case ISP_CLAMP: return i < 0 ? 0 : n - 1;
+    case ISP_MIRROR: return i < 0 ? -i - 1 : 2 * n - 1 - i;
+    case ISP_REPEAT: return i < 0 ? i + n : i - n;
+    default: return -1;
+    }
+}
+
 // Border tile staging: rows through the pattern once per row; 16-byte vectors whose columns
 // are all inside the image are copied as vectors, the rest byte by byte through the pattern
 // (the Body-tile launch requires w, h >= 2 tiles, so overshoots stay below N).
@@ -456,14 +463,14 @@ __device__ __noinline__ void stage_border(const Params &p, uint8_t *in, int x0, 
     constexpr int VPR = SW / 16;
     for (int k = threadIdx.x; k < SH * VPR; k += NT) {
         const int r = k / VPR, c = k % VPR;
-        const int yy = bmap(p.mode, y0 - 2 + r, p.h);          // -1: Constant, row outside
+        const int yy = bmap1(p.mode, y0 - 2 + r, p.h);         // -1: Constant, row outside
         uint8_t *dst = in + r * SW + 16 * c;
         const int xs = x0 - XO + 16 * c;
         if (yy >= 0 && xs >= 0 && xs + 16 <= p.w) {
             *reinterpret_cast<uint4 *>(dst) = __ldg(reinterpret_cast<const uint4 *>(p.img + (size_t)yy * p.pitch + xs));
         } else {
             for (int e = 0; e < 16; ++e) {
-                const int xx = bmap(p.mode, xs + e, p.w);
+                const int xx = bmap1(p.mode, xs + e, p.w);
                 dst[e] = (uint8_t)((yy < 0 || xx < 0) ? p.cval : p.img[(size_t)yy * p.pitch + xx]);
             }
         }
@@ -541,11 +548,14 @@ __global__ void __launch_bounds__(NT, FUSED_BODY_MINB) k_fused_body(const Params
 
     // ---- stage img rows y0-2 .. y0+TH+1, cols x0-16 .. x0+TW+15 -------------------------
     if (body) {
-        constexpr int VPR = SW / 16;
-        for (int k = tid; k < SH * VPR; k += NT) {
-            const int r = k / VPR, c = k % VPR;
-            const uint4 v = __ldg(reinterpret_cast<const uint4 *>(p.img + (size_t)(y0 - 2 + r) * p.pitch + x0 - XO) + c);
-            *reinterpret_cast<uint4 *>(&S.in[r][c * 16]) = v;
+        constexpr int VPR = SW / 16, DR = NT / VPR, DC = NT % VPR;   // (row, vector) stride per pass
+        int r = tid / VPR, c = tid % VPR;
+        const uint8_t *src = p.img + (size_t)(y0 - 2) * p.pitch + x0 - XO;
+        for (; r < SH;) {
+            *reinterpret_cast<uint4 *>(&S.in[r][c * 16]) = __ldg(reinterpret_cast<const uint4 *>(src + (size_t)r * p.pitch) + c);
+            r += DR;
+            c += DC;
+            if (c >= VPR) { c -= VPR; ++r; }
         }
     } else {
         stage_border(p, &S.in[0][0], x0, y0);
@@ -606,13 +616,24 @@ __global__ void __launch_bounds__(NT, FUSED_BODY_MINB) k_fused_body(const Params
         int H4[4];
         h5(r + 4, H4);
         const uint32_t cw = lw(S.in[r + 2] + XO + xr);
-        uint32_t lapw = 0;
+        // lap = clamp(box - 25 c, 0, 255) on 16-bit pair lanes: v = box + 25 (255 - c) is in
+        // [0, 12750]; clamp to [6375, 6630] (u16x2 max / min), subtract 6375
+        uint32_t bx_[4];
 #pragma unroll
         for (int k = 0; k < 4; ++k) {
-            const int v = H0[k] + H1[k] + H2[k] + H3[k] + H4[k] - 25 * (int)((cw >> (8 * k)) & 0xff);
-            lapw |= (uint32_t)min(255, max(0, v)) << (8 * k);
+            bx_[k] = (uint32_t)(H0[k] + H1[k] + H2[k] + H3[k] + H4[k]);
             H0[k] = H1[k]; H1[k] = H2[k]; H2[k] = H3[k]; H3[k] = H4[k];
         }
+        const uint32_t boxE = bx_[0] | bx_[2] << 16, boxO = bx_[1] | bx_[3] << 16;
+        const uint32_t cE = __byte_perm(cw, 0u, 0x4240), cO = __byte_perm(cw, 0u, 0x4341);
+        uint32_t vE = boxE + 25u * (0x00FF00FFu - cE), vO = boxO + 25u * (0x00FF00FFu - cO);
+        asm("max.u16x2 %0, %0, %1;" : "+r"(vE) : "r"(0x18E718E7u));   // 6375
+        asm("max.u16x2 %0, %0, %1;" : "+r"(vO) : "r"(0x18E718E7u));
+        asm("min.u16x2 %0, %0, %1;" : "+r"(vE) : "r"(0x19E619E6u));   // 6630
+        asm("min.u16x2 %0, %0, %1;" : "+r"(vO) : "r"(0x19E619E6u));
+        vE -= 0x18E718E7u;
+        vO -= 0x18E718E7u;
+        const uint32_t lapw = vE | vO << 8;          // lanes <= 255: bytes p0, p1, p2, p3
         // Harris (a10) on ext rows r, r+1, r+2 (image rows y-1, y, y+1)
         const HS c = hsum_row(S.fx[r + 2], S.fy[r + 2], G);
         const float2 two = f2(2.f, 2.f);
