@@ -8,6 +8,7 @@
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
+#include <functional>
 #include <mutex>
 #include <unordered_map>
 #include <vector>
@@ -505,17 +506,25 @@ isp_status_t resolve_and_launch(Desc &d, int fam, int w, int h, int mw, int mh, 
     const bool use_p = persist && sched != nullptr;
     const int tma_disp = (!direct && !use_p) ? DISP_TMA_STATIC : DISP_TMA;
     const int nwc = use_p ? pk.nwc : STAGED_WARPS;
-    const StagedGeom sg = staged_geom(w, hx, hy, px, esz, nin, nwc, use_p, pk.ring_kb);
+    StagedGeom sg = staged_geom(w, hx, hy, px, esz, nin, nwc, use_p, pk.ring_kb);
     if (direct) tma_ok = true;
     tma_ok = tma_ok && fn_of(tma_disp) != nullptr && g_override_wx == 0;
     const int tma_threads = direct ? TILE_THREADS : 32 * (nwc + 1);
-    const size_t tma_smem = direct ? (size_t)(TILE_PX * 32 + d.mw - 1) * (TILE_H + d.mh - 1) * esz : sg.smem;
+    size_t tma_smem = direct ? (size_t)(TILE_PX * 32 + d.mw - 1) * (TILE_H + d.mh - 1) * esz : sg.smem;
     const int nb_naive = blocks_per_sm(fn_of(naive_disp), threads);
     const int nb_stream = blocks_per_sm(fn_of(p0.wx > 1 ? DISP_WARP : DISP_BLOCK), threads);
     int nb_tma = tma_ok ? blocks_per_sm(fn_of(tma_disp), tma_threads, tma_smem) : 0;
     if (const char *e = getenv("ISP_CTAS_PER_SM")) nb_tma = std::min(nb_tma, std::max(1, atoi(e)));
     if (use_p) nb_tma = std::min(nb_tma, pk.ctas);
     if (tma_ok && nb_tma <= 0) tma_ok = false;
+    // static split with >= 8 resident CTAs / SM: a 3-slot ring per CTA (~50 KB of rows in
+    // flight per SM) measured 3 % faster than 4 on cfg2; fewer resident CTAs keep 4 slots
+    // (cfg5 7x7: 4 CTAs / SM, 3 slots measured slower) -- DESIGN.md 7b
+    if (tma_ok && !direct && !use_p && nb_tma >= 8 && sg.stages == 4 && sg.rs == 1 && !getenv("ISP_STAGES")) {
+        sg.stages = 3;
+        sg.smem = 512 + (size_t)3 * nin * sg.sw * esz;
+        tma_smem = sg.smem;
+    }
 
     // ISP_SPLIT (ablation of P:L90: one kernel per region instead of the fat kernel) plans
     // like ISP_BLOCK and launches each region's block rectangle separately
@@ -636,6 +645,43 @@ isp_status_t resolve_and_launch(Desc &d, int fam, int w, int h, int mw, int mh, 
     cudaError_t e = run(d);
     if (e == cudaSuccess) e = cudaGetLastError();
     return cuda_status(e, what);
+}
+
+// The tile-staged u8 / i16 kernels (tile_u8.cu) as the ISP_TMA variant of Laplace (which
+// = 0) and Harris (1): ISP_TMA runs them when eligible; ISP_AUTO evaluates Eq. (10) for
+// them (form S, reading A21, calibrated constants, occupancy from the API) against the
+// naive kernel.  Returns false when the caller should take the generic path.
+bool tile_variant(int which, int fam, int mode, int w, int h, int mw, int mh, isp_variant_t v, bool ok,
+                  const std::function<cudaError_t(int *)> &launch, isp_status_t &st, const char *what)
+{
+    if (!(v == ISP_TMA || v == ISP_AUTO) || !ok) return false;
+    int tw, th;
+    ispi_tile_shape(&tw, &th);
+    Plan p = make_plan(w, h, mw / 2, mh / 2, 4, tw, th, 128);
+    isp_plan_info info{};
+    n_block(p, info.n_block);
+    if (v == ISP_AUTO) {
+        isp_model_params mp;
+        defaults(fam, mode, mp);
+        mp.form = 2;
+        const int nb = ispi_tile_blocks_per_sm(which);
+        info.o_isp = occupancy_of(nb > 0 ? nb : 1, 128);
+        info.o_naive = 0.5;   // the naive streaming kernel (64 regs x 128 threads: 8 blocks / SM)
+        model(p, w, h, mw, mh, mp, info);
+        if (!(info.g > 1.0)) return false;
+    }
+    int b[4];
+    cudaError_t e = launch(b);
+    if (e == cudaSuccess) e = cudaGetLastError();
+    info.bh_l = b[0]; info.bh_r = b[1]; info.bh_t = b[2]; info.bh_b = b[3];
+    info.nx = p.nx; info.ny = p.ny;
+    info.degenerate = 0;
+    info.tile_w = tw; info.tile_h = th; info.warp_w = 128;
+    info.choice = ISP_TMA;
+    g_last_plan = info;
+    g_recent[g_n_plans++ % kRecent] = info;
+    st = cuda_status(e, what);
+    return true;
 }
 
 Desc base_desc(int w, int h, int pitch, int out_pitch, int mode, isp_stream_t stream)
@@ -1058,6 +1104,13 @@ isp_status_t isp_laplace5_u8(const uint8_t *img, int w, int h, int pitch, int bo
     if (const_val < 0 || const_val > 255) return fail(ISP_EINVAL, "u8 constant %d not in [0,255]", const_val);
     if (ranges_overlap(img, img_bytes(w, h, pitch, 1), out, img_bytes(w, h, out_pitch, 1)))
         return fail(ISP_EALIAS, "input and output overlap");
+    isp_status_t ts;
+    if (tile_variant(0, F_LAPLACE, border_mode, w, h, 5, 5, variant,
+                     ispi_tile_ok(img, nullptr, 1, w, h, pitch, out, out_pitch),
+                     [&](int *b) { return ispi_laplace_tile(img, w, h, pitch, border_mode, const_val, out, out_pitch,
+                                                            (cudaStream_t)stream, b); },
+                     ts, "isp_laplace5_u8(tile)"))
+        return ts;
     Desc d = base_desc(w, h, pitch, out_pitch, border_mode, stream);
     d.in0 = img;
     d.out0 = out;
@@ -1083,6 +1136,12 @@ isp_status_t isp_harris_u8(const int16_t *dx, const int16_t *dy, int w, int h, i
     const size_t ob = img_bytes(w, h, out_pitch, 1);
     if (ranges_overlap(dx, img_bytes(w, h, pitch, 2), out, ob) || ranges_overlap(dy, img_bytes(w, h, pitch, 2), out, ob))
         return fail(ISP_EALIAS, "input and output overlap");
+    isp_status_t ts;
+    if (tile_variant(1, F_HARRIS, border_mode, w, h, 3, 3, variant, ispi_tile_ok(dx, dy, 2, w, h, pitch, out, out_pitch),
+                     [&](int *b) { return ispi_harris_tile(dx, dy, w, h, pitch, border_mode, const_val, thr, out,
+                                                           out_pitch, (cudaStream_t)stream, b); },
+                     ts, "isp_harris_u8(tile)"))
+        return ts;
     Desc d = base_desc(w, h, pitch, out_pitch, border_mode, stream);
     d.in0 = dx;
     d.in1 = dy;

@@ -24,3 +24,13 @@ isp_status_t ispi_filter_u8(const uint8_t *img, int w, int h, int pitch, const i
                             isp_variant_t variant, isp_stream_t stream, const RowRange *rr);
 isp_status_t ispi_filter_tex_f32(const float *img, int w, int h, int pitch, const float *mask, int mw, int mh,
                                  int border_mode, float const_val, float *out, int out_pitch, isp_stream_t stream);
+
+// tile-staged u8 / i16 kernels (tile_u8.cu): the ISP_TMA variant of Laplace and Harris
+#include <cuda_runtime.h>
+bool ispi_tile_ok(const void *in0, const void *in1, int elem, int w, int h, int pitch, const void *out, int out_pitch);
+void ispi_tile_shape(int *tw, int *th);
+int ispi_tile_blocks_per_sm(int which);
+cudaError_t ispi_laplace_tile(const uint8_t *img, int w, int h, int pitch, int mode, int cval, uint8_t *out,
+                              int out_pitch, cudaStream_t st, int bounds[4]);
+cudaError_t ispi_harris_tile(const int16_t *dx, const int16_t *dy, int w, int h, int pitch, int mode, int cval,
+                             long long thr, uint8_t *out, int out_pitch, cudaStream_t st, int bounds[4]);

@@ -18,7 +18,10 @@
 
 namespace ispk {
 
-constexpr int kStagedComputeWarps = 4;
+#ifndef ISP_STAGED_WARPS
+#define ISP_STAGED_WARPS 4
+#endif
+constexpr int kStagedComputeWarps = ISP_STAGED_WARPS;
 constexpr int kStagedThreads = 32 * (kStagedComputeWarps + 1);
 constexpr int kStagedMaxStages = 32;
 constexpr int kStagedBarrierBytes = 512;  // full[32] + empty[32] mbarriers

@@ -65,7 +65,10 @@ cudaError_t run_bilateral(const Desc &);
 
 // pixels per thread (x) of each family
 constexpr int PX_F32 = 4, PX_U8 = kPxU8, PX_I16 = kPxI16, PX_DIRECT = 4;
-constexpr int STAGED_WARPS = 4, STAGED_THREADS = 160;
+#ifndef ISP_STAGED_WARPS
+#define ISP_STAGED_WARPS 4
+#endif
+constexpr int STAGED_WARPS = ISP_STAGED_WARPS, STAGED_THREADS = 32 * (ISP_STAGED_WARPS + 1);
 // shared-memory tiled kernel of the runtime-window ops (isp_direct.cuh k_tile)
 constexpr int TILE_THREADS = 256, TILE_H = 16, TILE_PX = 4;
 

@@ -475,3 +475,34 @@ def test_peer_strips_u8(isp, nranks):
                 got[y0:y0 + sh] = host(isp.isp_shard_filter_peer_local_u8(strips[r], prev, nxt, H, r, nranks, mask,
                                                                           div, mode, 9, variant=v))
             np.testing.assert_array_equal(got, ref, err_msg=f"{mode} {v} P={nranks}")
+
+
+# ---------------------------------------------------------------- tile-staged Laplace / Harris
+@pytest.mark.parametrize("shape", [(260, 2064), (133, 400), (4096 // 8, 4096)])
+def test_laplace_harris_tile_kernels(isp, shape):
+    """The tile-staged ISP kernels of Laplace and Harris (tile_u8.cu; Body tiles unchecked,
+    border tiles staged through the pattern, partial right / bottom tiles): bit-exact
+    against the oracle in every mode, several Harris thresholds, the plan showing the
+    tile variant (choice TMA, 128 x 32 tiles)."""
+    h, w = shape
+    img = synth.structured_u8(h, w, 12)
+    d = dev(img)
+    for mode in MODES:
+        rlap = oracle.laplace5_u8(img, mode, 33)
+        got = host(isp.isp_laplace5_u8(d, mode, 33, variant="tma"))
+        p = isp.isp_last_plan()
+        assert p["choice"] == CODE["tma"] and p["tile_w"] == 128 and p["tile_h"] == 32, p
+        np.testing.assert_array_equal(got, rlap, err_msg=f"laplace {mode}")
+        rdx, rdy, _ = oracle.sobel(img, mode, 33)
+        ddx, ddy = dev(rdx), dev(rdy)
+        c = 700 if mode == "constant" else 0
+        for thr in (0, -(10 ** 7), 10 ** 9, 10 ** 12):
+            rhar = oracle.harris(rdx, rdy, mode, c, thr)
+            got = host(isp.isp_harris_u8(ddx, ddy, mode, c, thr, variant="tma"))
+            assert isp.isp_last_plan()["choice"] == CODE["tma"]
+            np.testing.assert_array_equal(got, rhar, err_msg=f"harris {mode} thr={thr}")
+        # random int16 derivatives over the whole Sobel range
+        rx = synth.random_i16(h, w, 5)
+        ry = synth.random_i16(h, w, 6)
+        np.testing.assert_array_equal(host(isp.isp_harris_u8(dev(rx), dev(ry), mode, -3, 10 ** 11, variant="tma")),
+                                      oracle.harris(rx, ry, mode, -3, 10 ** 11), err_msg=f"harris random {mode}")

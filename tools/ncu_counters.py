@@ -113,6 +113,30 @@ def inner(a):
     json.dump(labels, open(a.labels, "w"))
 
 
+def markdown(out, tag):
+    """Table I / Table II analog: per launch, per output pixel."""
+    lines = [f"# ncu counters {tag}: ISP vs naive (Table I / II analog), one launch per row",
+             "", "Per output pixel: thread instructions, branch instructions (thread-level), predicated-on share; "
+             "registers, register occupancy limit (blocks / SM), achieved warps. `tools/ncu_counters.py`.", "",
+             "| case | us | inst/px | branch/px | pred-on % | divergent branches | regs | occ. limit (regs) | warps active % |",
+             "|---|---|---|---|---|---|---|---|---|"]
+    for r in out["records"]:
+        px = r["px"]
+        ti = r["smsp__thread_inst_executed.sum"]
+        lines.append("| {} | {:.1f} | {:.1f} | {:.2f} | {:.1f} | {:.0f} | {:.0f} | {:.0f} | {:.1f} |".format(
+            r["label"], r["gpu__time_duration.sum"] / 1000.0, ti / px,
+            r["smsp__sass_inst_executed_op_branch.sum"] * 32 / px,
+            100.0 * r["smsp__thread_inst_executed_pred_on.sum"] / ti, r["smsp__sass_branch_targets_threads_divergent.sum"],
+            r["launch__registers_per_thread"], r["launch__occupancy_limit_registers"],
+            r["sm__warps_active.avg.pct_of_peak_sustained_active"]))
+    lines += ["", "## Calibration (reading A19): n_kernel = I_isp / (m n px), n_check = (I_naive - I_isp) / (4 m n px)",
+              "", "| family / mode | n_check | n_kernel | inst/px ISP | inst/px naive |", "|---|---|---|---|---|"]
+    for k, v in sorted(out["calibration"].items()):
+        lines.append(f"| {k} | {v['n_check']:.4f} | {v['n_kernel']:.4f} | {v['thread_inst_per_px_isp']:.1f} | "
+                     f"{v['thread_inst_per_px_naive']:.1f} |")
+    return "\n".join(lines) + "\n"
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--tag", default="r02")
@@ -167,6 +191,7 @@ def main():
     out = {"records": res, "calibration": cal, "metrics": METRICS}
     path = os.path.join(a.out_dir, f"{a.tag}_counters.json")
     json.dump(out, open(path, "w"), indent=1)
+    open(path[:-5] + ".md", "w").write(markdown(out, a.tag))
     print(f"wrote {path}: {len(res)} records, {len(cal)} calibration rows")
     if r.returncode != 0:
         print(r.stderr[-3000:], file=sys.stderr)
