@@ -407,6 +407,11 @@ def run_isp(args):
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     with ClockSampler(local) as cs:
         t_wall0 = time.time()
+        # keep the GPU busy (~2 ms spin, before the start event) while the host enqueues
+        # the start event, the K-step graph and the stop event: the timed region is then
+        # exactly the K steps on the device, not the host's graph-launch latency
+        with torch.cuda.stream(stream):
+            torch.cuda._sleep(4_000_000)
         e0.record(stream)
         run_steps(args.steps)
         e1.record(stream)
@@ -434,8 +439,9 @@ def run_isp(args):
     roof = {"bound": "hbm", "achieved": achieved, "peak": hbm if hbm else 6650.0, "unit": "GB/s",
             "frac": achieved / (hbm if hbm else 6650.0),
             "peak_source": "MEASURED_PEAKS.json hbm_gbs (measured)" if hbm else "fallback (B200_PROFILING.md)",
-            "kernel": f"variant {args.variant}: " + (f"k_pstaged<{kname}> (TMA-staged ISP)" if plan["choice"] == 4
-                                                     else f"k_stencil<{kname}>"),
+            "kernel": f"variant {args.variant}: " + (
+                (f"k_pstaged<{kname}> (persistent TMA-staged ISP)" if os.environ.get("ISP_TMA_PERSIST") == "1"
+                 else f"k_staged<{kname}> (TMA-staged ISP)") if plan["choice"] == 4 else f"k_stencil<{kname}>"),
             "algorithmic_bytes_per_launch": rank_bytes,
             "duration_us": per_launch_us,
             "duration_method": "timed region / launches (one CUDA graph of the K steps, kernels back to back)"}
@@ -461,6 +467,7 @@ def run_isp(args):
                 a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
                 with torch.cuda.stream(stream):
                     g.replay()
+                    torch.cuda._sleep(2_000_000)
                     a.record(stream)
                     for _ in range(reps):
                         g.replay()
