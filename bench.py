@@ -315,7 +315,11 @@ def run_isp(args):
     if world > 1 and halo_path == "peer":
         try:
             own = [pairs[k][0][halo:halo + sh] for k in range(npairs)]
-            peers = [isp.isp_shard_peer_open(ctx, o, ring=True) for o in own]
+            peers = []
+            for o in own:   # CUDA IPC handles of every rank's strip, exchanged over the process group
+                hs = [None] * world
+                dist.all_gather_object(hs, isp.isp_shard_peer_handle(o))
+                peers.append(isp.isp_shard_peer_attach(rank, world, o, hs, ring=True))
             ok = torch.tensor([1.0], device=dev)
         except Exception as e:   # no IPC in this environment: fall back to the NCCL exchange
             print(f"[bench] rank {rank}: peer open failed ({e}); using the NCCL halo exchange", file=sys.stderr)

@@ -277,6 +277,12 @@ isp_status_t isp_shard_exchange(isp_shard_ctx *ctx, void *strip, int elem_size, 
  * f32 and u8 filters (isp_filter_ex / isp_filter_u8 semantics, all variants except TEX). */
 typedef struct isp_shard_peer isp_shard_peer;
 isp_status_t isp_shard_peer_open(isp_shard_ctx *ctx, void *strip, int ring, isp_shard_peer **out);
+/* The two halves of isp_shard_peer_open for callers that exchange the 72-byte handles
+ * themselves (e.g. over a gloo process group): the handle of this rank's strip, and the
+ * attach of the neighbours given every rank's handle (nranks x 72 bytes, rank order). */
+isp_status_t isp_shard_peer_handle(void *strip, unsigned char out[72]);
+isp_status_t isp_shard_peer_attach(int rank, int nranks, int device, void *strip, const unsigned char *handles,
+                                   int ring, isp_shard_peer **out);
 isp_status_t isp_shard_peer_filter_f32(isp_shard_peer *peer, int w, int H, int pitch, const float *mask, int mw,
                                        int mh, int border_mode, float const_val, float *out, int out_pitch,
                                        isp_variant_t variant, isp_stream_t stream);

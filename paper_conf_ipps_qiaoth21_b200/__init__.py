@@ -31,6 +31,7 @@ __all__ = [
     "isp_shard_filter_f32", "isp_shard_filter_u8", "isp_shard_filter_local_f32", "isp_shard_filter_local_u8",
     "isp_shard_exchange", "isp_shard_destroy", "isp_shard_peer_open", "isp_shard_peer_filter_f32",
     "isp_shard_peer_close", "isp_shard_filter_peer_local_f32", "isp_shard_filter_peer_local_u8",
+    "isp_shard_peer_handle", "isp_shard_peer_attach",
 ]
 
 CLAMP, MIRROR, REPEAT, CONSTANT = 0, 1, 2, 3
@@ -122,6 +123,8 @@ _SIGS = {
     "isp_shard_peer_open": [_P, _P, _I, _P],
     "isp_shard_peer_filter_f32": [_P, _I, _I, _I, _P, _I, _I, _I, _F, _P, _I, _I, _P],
     "isp_shard_peer_close": [_P],
+    "isp_shard_peer_handle": [_P, _P],
+    "isp_shard_peer_attach": [_I, _I, _I, _P, _P, _I, _P],
     "isp_shard_filter_peer_local_f32": [_P, _P, _P, _I, _I, _I, _I, _I, _P, _I, _I, _I, _F, _P, _I, _I, _P],
     "isp_shard_filter_peer_local_u8": [_P, _P, _P, _I, _I, _I, _I, _I, _P, _I, _I, ctypes.c_int32, _I, _I, _P, _I,
                                        _I, _P],
@@ -586,9 +589,30 @@ def isp_shard_peer_open(ctx, strip, ring=True):
 _PEER_CTX = {}
 
 
+def isp_shard_peer_handle(strip) -> bytes:
+    """72-byte CUDA IPC handle (+ offset) of a strip's allocation, for isp_shard_peer_attach."""
+    buf = (ctypes.c_ubyte * 72)()
+    _check(lib().isp_shard_peer_handle(strip.data_ptr(), buf))
+    return bytes(buf)
+
+
+def isp_shard_peer_attach(rank, nranks, strip, handles, ring=True, device=None):
+    """Map the neighbour strips from every rank's handle (list of 72-byte blobs, rank order)."""
+    dev_i = strip.device.index if device is None else int(device)
+    blob = b"".join(handles)
+    if len(blob) != 72 * int(nranks):
+        raise ValueError("need one 72-byte handle per rank")
+    buf = (ctypes.c_ubyte * len(blob)).from_buffer_copy(blob)
+    pp = ctypes.c_void_p()
+    _check(lib().isp_shard_peer_attach(int(rank), int(nranks), dev_i, strip.data_ptr(), buf, int(bool(ring)),
+                                       ctypes.byref(pp)))
+    _PEER_CTX[pp.value] = ((int(rank), int(nranks)), strip)
+    return pp
+
+
 def isp_shard_peer_filter_f32(pp, H, mask, border_mode, const_val=0.0, out=None, variant=AUTO, w=None, stream=None):
     ctx, strip = _PEER_CTX[pp.value]
-    rank, nranks = _ctx_ranks(ctx, None, None)
+    rank, nranks = ctx if isinstance(ctx, tuple) else _ctx_ranks(ctx, None, None)
     sh = _own_strip(strip, torch.float32, H, rank, nranks)
     w, _, pitch = _geom(strip, w)
     m, mp = _host(mask, ctypes.c_float)

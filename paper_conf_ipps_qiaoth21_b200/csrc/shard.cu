@@ -313,25 +313,25 @@ isp_status_t isp_shard_filter_peer_local_u8(const uint8_t *own, const uint8_t *p
 }  // extern "C"
 
 struct isp_shard_peer {
-    isp_shard_ctx *ctx;
+    int rank, nranks, device;
     void *own;
     void *prev, *next;        // neighbour strips (opened IPC mappings), or null
     void *prev_base, *next_base;
 };
 
 namespace {
-struct PeerInfo {
+struct PeerInfo {                    // 72 bytes: IPC handle of the allocation + offset
     cudaIpcMemHandle_t h;
     unsigned long long off;
 };
+static_assert(sizeof(PeerInfo) == 72, "peer handle layout");
 }  // namespace
 
 extern "C" {
 
-isp_status_t isp_shard_peer_open(isp_shard_ctx *ctx, void *strip, int ring, isp_shard_peer **out)
+isp_status_t isp_shard_peer_handle(void *strip, unsigned char out[72])
 {
-    if (!ctx || !strip || !out) return ispi_fail(ISP_EINVAL, "isp_shard_peer_open args");
-    if (cudaSetDevice(ctx->device) != cudaSuccess) return ispi_fail(ISP_ECUDA, "cudaSetDevice");
+    if (!strip || !out) return ispi_fail(ISP_EINVAL, "isp_shard_peer_handle args");
     // allocation base of the strip (IPC handles name allocations; torch's caching
     // allocator hands out sub-ranges): cuMemGetAddressRange through the runtime's driver
     // entry point, so libisp.so does not link libcuda (CPU boxes load it without a driver)
@@ -348,6 +348,59 @@ isp_status_t isp_shard_peer_open(isp_shard_ctx *ctx, void *strip, int ring, isp_
     cudaError_t e = cudaIpcGetMemHandle(&mine.h, (void *)base);
     if (e != cudaSuccess) return ispi_fail(ISP_ECUDA, "cudaIpcGetMemHandle: %s", cudaGetErrorString(e));
     mine.off = (unsigned long long)((CUdeviceptr)strip - base);
+    std::memcpy(out, &mine, sizeof(mine));
+    return ISP_OK;
+}
+
+isp_status_t isp_shard_peer_attach(int rank, int nranks, int device, void *strip, const unsigned char *handles,
+                                   int ring, isp_shard_peer **out)
+{
+    if (!strip || !handles || !out || nranks < 1 || rank < 0 || rank >= nranks)
+        return ispi_fail(ISP_EINVAL, "isp_shard_peer_attach args");
+    if (cudaSetDevice(device) != cudaSuccess) return ispi_fail(ISP_ECUDA, "cudaSetDevice(%d)", device);
+    std::vector<PeerInfo> all(nranks);
+    std::memcpy(all.data(), handles, sizeof(PeerInfo) * nranks);
+    isp_shard_peer *pp = new isp_shard_peer{};
+    pp->rank = rank;
+    pp->nranks = nranks;
+    pp->device = device;
+    pp->own = strip;
+    const int P = nranks, r = rank;
+    const int pr = r > 0 ? r - 1 : ((ring && P > 1) ? P - 1 : -1);
+    const int nx = r < P - 1 ? r + 1 : ((ring && P > 1) ? 0 : -1);
+    auto open = [&](int q, void *&basep, void *&ptr) -> isp_status_t {
+        if (q < 0 || q == r) return ISP_OK;
+        cudaError_t ee = cudaIpcOpenMemHandle(&basep, all[q].h, cudaIpcMemLazyEnablePeerAccess);
+        if (ee != cudaSuccess) {
+            cudaGetLastError();
+            return ispi_fail(ISP_ECUDA, "cudaIpcOpenMemHandle(rank %d): %s", q, cudaGetErrorString(ee));
+        }
+        ptr = (char *)basep + all[q].off;
+        return ISP_OK;
+    };
+    isp_status_t s = open(pr, pp->prev_base, pp->prev);
+    if (s == ISP_OK) {
+        if (nx == pr && nx >= 0) {   // P = 2 ring: one mapping serves both sides
+            pp->next = pp->prev;
+        } else {
+            s = open(nx, pp->next_base, pp->next);
+        }
+    }
+    if (s != ISP_OK) {
+        isp_shard_peer_close(pp);
+        return s;
+    }
+    *out = pp;
+    return ISP_OK;
+}
+
+isp_status_t isp_shard_peer_open(isp_shard_ctx *ctx, void *strip, int ring, isp_shard_peer **out)
+{
+    if (!ctx || !strip || !out) return ispi_fail(ISP_EINVAL, "isp_shard_peer_open args");
+    if (cudaSetDevice(ctx->device) != cudaSuccess) return ispi_fail(ISP_ECUDA, "cudaSetDevice");
+    PeerInfo mine{};
+    isp_status_t s = isp_shard_peer_handle(strip, reinterpret_cast<unsigned char *>(&mine));
+    if (s != ISP_OK) return s;
     const int P = ctx->nranks;
     PeerInfo *dsend = nullptr, *drecv = nullptr;
     std::vector<PeerInfo> all(P);
@@ -356,33 +409,15 @@ isp_status_t isp_shard_peer_open(isp_shard_ctx *ctx, void *strip, int ring, isp_
         cudaStreamCreate(&st) != cudaSuccess)
         return ispi_fail(ISP_ECUDA, "peer handle exchange buffers");
     cudaMemcpy(dsend, &mine, sizeof(PeerInfo), cudaMemcpyHostToDevice);
-    isp_status_t s = nccl_status(ncclAllGather(dsend, drecv, sizeof(PeerInfo), ncclUint8, ctx->comm, st),
-                                 "ncclAllGather(ipc handles)");
+    s = nccl_status(ncclAllGather(dsend, drecv, sizeof(PeerInfo), ncclUint8, ctx->comm, st), "ncclAllGather(ipc handles)");
     if (s == ISP_OK && cudaStreamSynchronize(st) != cudaSuccess) s = ispi_fail(ISP_ECUDA, "handle exchange");
     if (s == ISP_OK) cudaMemcpy(all.data(), drecv, sizeof(PeerInfo) * P, cudaMemcpyDeviceToHost);
     cudaFree(dsend);
     cudaFree(drecv);
     cudaStreamDestroy(st);
     if (s != ISP_OK) return s;
-    isp_shard_peer *pp = new isp_shard_peer{};
-    pp->ctx = ctx;
-    pp->own = strip;
-    const int r = ctx->rank;
-    const int pr = r > 0 ? r - 1 : ((ring && P > 1) ? P - 1 : -1);
-    const int nx = r < P - 1 ? r + 1 : ((ring && P > 1) ? 0 : -1);
-    auto open = [&](int q, void *&basep, void *&ptr) -> isp_status_t {
-        if (q < 0 || q == r) return ISP_OK;
-        cudaError_t ee = cudaIpcOpenMemHandle(&basep, all[q].h, cudaIpcMemLazyEnablePeerAccess);
-        if (ee != cudaSuccess) return ispi_fail(ISP_ECUDA, "cudaIpcOpenMemHandle(rank %d): %s", q, cudaGetErrorString(ee));
-        ptr = (char *)basep + all[q].off;
-        return ISP_OK;
-    };
-    if ((s = open(pr, pp->prev_base, pp->prev)) != ISP_OK || (s = open(nx, pp->next_base, pp->next)) != ISP_OK) {
-        isp_shard_peer_close(pp);
-        return s;
-    }
-    *out = pp;
-    return ISP_OK;
+    return isp_shard_peer_attach(ctx->rank, P, ctx->device, strip, reinterpret_cast<const unsigned char *>(all.data()),
+                                 ring, out);
 }
 
 isp_status_t isp_shard_peer_filter_f32(isp_shard_peer *pp, int w, int H, int pitch, const float *mask, int mw, int mh,
@@ -390,10 +425,10 @@ isp_status_t isp_shard_peer_filter_f32(isp_shard_peer *pp, int w, int H, int pit
                                        isp_variant_t variant, isp_stream_t stream)
 {
     if (!pp) return ispi_fail(ISP_EINVAL, "null peer context");
-    if (cudaSetDevice(pp->ctx->device) != cudaSuccess) return ispi_fail(ISP_ECUDA, "cudaSetDevice");
+    if (cudaSetDevice(pp->device) != cudaSuccess) return ispi_fail(ISP_ECUDA, "cudaSetDevice");
     return isp_shard_filter_peer_local_f32((const float *)pp->own, (const float *)pp->prev, (const float *)pp->next, w,
-                                           H, pitch, pp->ctx->rank, pp->ctx->nranks, mask, mw, mh, border_mode,
-                                           const_val, out, out_pitch, variant, stream);
+                                           H, pitch, pp->rank, pp->nranks, mask, mw, mh, border_mode, const_val, out,
+                                           out_pitch, variant, stream);
 }
 
 isp_status_t isp_shard_peer_close(isp_shard_peer *pp)
