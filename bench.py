@@ -267,10 +267,21 @@ def run_isp(args):
     import synth
 
     rank, world, local = env_rank()
+    # ISP_BENCH_SAME_DEVICE=1 (test hook): every rank on cuda:0 with a gloo process group
+    # and the peer path only -- the multi-rank code on a one-GPU box (CUDA IPC works between
+    # processes on one device; NCCL does not take two ranks per device)
+    same_dev = os.environ.get("ISP_BENCH_SAME_DEVICE") == "1" and world > 1
+    if same_dev:
+        local = 0
+        args.halo = "peer"
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
+    rdev = torch.device("cpu") if same_dev else dev      # device of the reduction tensors
     if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        if same_dev:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=dev)
     isp.lib()
     wl = Workload(args.workload, world)
     mask = wl.mask()
@@ -301,7 +312,7 @@ def run_isp(args):
         pairs.append((inp, out))
     ctx = None
     comm_stream = torch.cuda.Stream(device=dev)
-    if world > 1:
+    if world > 1 and not same_dev:
         uid = [isp.isp_shard_unique_id() if rank == 0 else None]
         dist.broadcast_object_list(uid, src=0)
         ctx = isp.isp_shard_init(uid[0], rank, world, local)
@@ -320,16 +331,17 @@ def run_isp(args):
                 hs = [None] * world
                 dist.all_gather_object(hs, isp.isp_shard_peer_handle(o))
                 peers.append(isp.isp_shard_peer_attach(rank, world, o, hs, ring=True))
-            ok = torch.tensor([1.0], device=dev)
+            ok = torch.tensor([1.0], device=rdev)
         except Exception as e:   # no IPC in this environment: fall back to the NCCL exchange
             print(f"[bench] rank {rank}: peer open failed ({e}); using the NCCL halo exchange", file=sys.stderr)
-            ok = torch.tensor([0.0], device=dev)
+            ok = torch.tensor([0.0], device=rdev)
         dist.all_reduce(ok, op=dist.ReduceOp.MIN)
         if ok.item() < 1:
             if peers:
                 for pp in peers:
                     isp.isp_shard_peer_close(pp)
             peers, halo_path = None, "nccl (peer open failed)"
+        torch.cuda.synchronize()
         dist.barrier()      # every strip holds its data before any rank reads a neighbour's
 
     def launch(mode, pair, v=variant):
@@ -425,7 +437,7 @@ def run_isp(args):
         dist.barrier()
     ms = e0.elapsed_time(e1)
     if world > 1:
-        t = torch.tensor([ms], device=dev)
+        t = torch.tensor([ms], device=rdev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         ms = float(t.item())
     clocks = cs.summary(t_wall0, t_wall1)
@@ -485,7 +497,7 @@ def run_isp(args):
 
     # ---- halo exchange alone (N > 1): NCCL send/recv of the strip edges on the comm stream ----
     halo_us = None
-    if world > 1:
+    if world > 1 and ctx is not None:
         inp = pairs[0][0]
         R = 50
         dist.barrier()
@@ -497,13 +509,13 @@ def run_isp(args):
                 isp.isp_shard_exchange(ctx, inp, H_img, halo, halo, modes[-1], comm_stream=comm_stream)
             b.record(comm_stream)
         torch.cuda.synchronize()
-        t = torch.tensor([a.elapsed_time(b) * 1e3 / R], device=dev)
+        t = torch.tensor([a.elapsed_time(b) * 1e3 / R], device=rdev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         halo_us = float(t.item())
 
     # ---- end to end: pinned host buffers, H2D + filter + D2H inside the timed region ----
     e2e = None
-    if not args.quick:
+    if not args.quick and not same_dev:
         hin = (torch.from_numpy(host_img) if host_img is not None else src).pin_memory()
         houts = [torch.empty((sh, W), dtype=torch.float32).pin_memory() for _ in range(2)]
         E = max(3, min(20, args.steps // 100)) if wl.name == "cfg2" else 3
@@ -528,7 +540,7 @@ def run_isp(args):
         torch.cuda.synchronize()
         ems = a.elapsed_time(b)
         if world > 1:
-            t = torch.tensor([ems], device=dev)
+            t = torch.tensor([ems], device=rdev)
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
             ems = float(t.item())
         e2e = {"value": px_step * E / (ems / 1e3) / 1e6, "unit": UNIT,

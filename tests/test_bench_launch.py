@@ -36,3 +36,22 @@ def test_world_size_mismatch_is_an_error():
     r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--gpus", "4", "--check-launch"],
                        capture_output=True, text=True, timeout=300, cwd=ROOT, env=env)
     assert r.returncode != 0 and "WORLD_SIZE" in r.stderr
+
+
+@pytest.mark.gpu
+def test_bench_two_ranks_peer_path_one_gpu():
+    """bench.py --gpus 2 end to end on a one-GPU box: the test hook ISP_BENCH_SAME_DEVICE=1
+    puts both ranks on cuda:0 (gloo process group, CUDA IPC between the processes), so the
+    multi-rank code -- handle exchange, peer-direct strip launches, graphs, max-over-ranks
+    timing -- runs before a multi-GPU box is available (the numbers are not a measurement)."""
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    env = dict(os.environ, ISP_BENCH_SAME_DEVICE="1")
+    env.pop("WORLD_SIZE", None)
+    r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--gpus", "2", "--steps", "3", "--warmup", "3",
+                        "--quick", "--no-cpu"], capture_output=True, text=True, timeout=900, cwd=ROOT, env=env)
+    assert r.returncode == 0, r.stderr[-3000:]
+    d = _json_lines(r.stdout)[-1]
+    assert d["n_gpus"] == 2 and d["halo_path"] == "peer" and d["gpu_launches"] == 3 * 4
+    assert d["config"]["image"] == [8192, 4096] and d["value"] > 0
