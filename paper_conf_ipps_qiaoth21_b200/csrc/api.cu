@@ -651,20 +651,22 @@ isp_status_t resolve_and_launch(Desc &d, int fam, int w, int h, int mw, int mh, 
 // = 0) and Harris (1): ISP_TMA runs them when eligible; ISP_AUTO evaluates Eq. (10) for
 // them (form S, reading A21, calibrated constants, occupancy from the API) against the
 // naive kernel.  Returns false when the caller should take the generic path.
+// which = 2: the Laplace band kernel (band_u8.cu: warp strips of 256 columns x bands of rows)
 bool tile_variant(int which, int fam, int mode, int w, int h, int mw, int mh, isp_variant_t v, bool ok,
                   const std::function<cudaError_t(int *)> &launch, isp_status_t &st, const char *what)
 {
     if (!(v == ISP_TMA || v == ISP_AUTO) || !ok) return false;
     int tw, th;
-    ispi_tile_shape(&tw, &th);
-    Plan p = make_plan(w, h, mw / 2, mh / 2, 4, tw, th, 128);
+    if (which == 2) ispi_band_shape(w, h, &tw, &th);
+    else ispi_tile_shape(&tw, &th);
+    Plan p = make_plan(w, h, mw / 2, mh / 2, 4, tw, th, which == 2 ? 256 : 128);
     isp_plan_info info{};
     n_block(p, info.n_block);
     if (v == ISP_AUTO) {
         isp_model_params mp;
         defaults(fam, mode, mp);
         mp.form = 2;
-        const int nb = ispi_tile_blocks_per_sm(which);
+        const int nb = which == 2 ? ispi_band_blocks_per_sm() : ispi_tile_blocks_per_sm(which);
         info.o_isp = occupancy_of(nb > 0 ? nb : 1, 128);
         info.o_naive = 0.5;   // the naive streaming kernel (64 regs x 128 threads: 8 blocks / SM)
         model(p, w, h, mw, mh, mp, info);
@@ -676,7 +678,7 @@ bool tile_variant(int which, int fam, int mode, int w, int h, int mw, int mh, is
     info.bh_l = b[0]; info.bh_r = b[1]; info.bh_t = b[2]; info.bh_b = b[3];
     info.nx = p.nx; info.ny = p.ny;
     info.degenerate = 0;
-    info.tile_w = tw; info.tile_h = th; info.warp_w = 128;
+    info.tile_w = tw; info.tile_h = th; info.warp_w = which == 2 ? 256 : 128;
     info.choice = ISP_TMA;
     g_last_plan = info;
     g_recent[g_n_plans++ % kRecent] = info;
@@ -1105,6 +1107,12 @@ isp_status_t isp_laplace5_u8(const uint8_t *img, int w, int h, int pitch, int bo
     if (ranges_overlap(img, img_bytes(w, h, pitch, 1), out, img_bytes(w, h, out_pitch, 1)))
         return fail(ISP_EALIAS, "input and output overlap");
     isp_status_t ts;
+    // ISP_TMA / AUTO: the band kernel (band_u8.cu) when eligible, else the tile kernel
+    if (tile_variant(2, F_LAPLACE, border_mode, w, h, 5, 5, variant, ispi_band_ok(img, w, h, pitch, out, out_pitch),
+                     [&](int *b) { return ispi_laplace_band(img, w, h, pitch, border_mode, const_val, out, out_pitch,
+                                                            (cudaStream_t)stream, b); },
+                     ts, "isp_laplace5_u8(band)"))
+        return ts;
     if (tile_variant(0, F_LAPLACE, border_mode, w, h, 5, 5, variant,
                      ispi_tile_ok(img, nullptr, 1, w, h, pitch, out, out_pitch),
                      [&](int *b) { return ispi_laplace_tile(img, w, h, pitch, border_mode, const_val, out, out_pitch,

@@ -1,0 +1,420 @@
+// band_u8.cu -- warp-strip streaming ISP kernels for the cfg3 u8 operators (round 3): the
+// ISP_TMA variant of isp_laplace5_u8 (a8).
+//
+// Partition (Listing 3, at warp granularity as in Listing 5): the
+// image is cut into vertical strips of 32 lanes x 4*NW pixels (one warp each; NW = 2 or 4 words) and horizontal
+// bands of rows (balanced over one wave of CTAs).  A warp's region follows from whether
+// its strip reaches past the left / right edge and its band past the top / bottom edge
+// within the window's reach -- warp-uniform -- so every warp runs a body specialised to
+// exactly those checks ("fat kernel"); Body warps run none.
+//
+// Each warp streams the input rows of its band through its own shared-memory ring with
+// cp.async (4*NW bytes per lane; the strip's two 4-byte halo words by lanes 0 and 31,
+// predicated), D rows
+// in flight, and keeps the per-row horizontal 5-sums in a register ring:
+//   * horizontal 5-sums directly as 16-bit pair lanes: with E_k = (b_k, b_k+2) and
+//     O_k = (b_k+1, b_k+3) (byte permutes of the lane's words and funnel shifts across them),
+//     (H0, H2) = S + E_-2 and (H1, H3) = S + O_2 with S = O_-2 + E_0 + O_0 + E_2;
+//   * the 5-row box as a running sum on 16-bit pair lanes (pixels (0,2) / (1,3) of each
+//     4-pixel group), biased by 6400 = 0x1900 so that clamp(box - 25 c, 0, 255) is a
+//     u16x2 max / min against 0x1900 / 0x19FF and the result is the low byte of each lane.
+// Border handling lives only in the region bodies: T / B warps map their out-of-image
+// rows through the pattern once per row (Constant: the row is C), L / R warps fix the two
+// halo bytes beyond the edge in registers (Repeat: the edge lane copies the wrapped word).
+// Results are the oracle's bit for bit (exact integer arithmetic).
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <algorithm>
+#include <cstdlib>
+
+#include "../../include/isp.h"
+#include "internal.h"
+
+namespace {
+
+constexpr int BW = 4;                      // warps per CTA (adjacent strips of one band)
+constexpr int NTB = 32 * BW;
+#ifndef BAND_LAP_D
+#define BAND_LAP_D 5
+#endif
+constexpr int LD = BAND_LAP_D;             // rows in flight per warp
+constexpr int LR = 8;                      // ring slots (power of 2): newest + D in flight
+static_assert(LR >= LD + 1, "ring too small");
+
+// NW words (4 pixels each) per lane
+template <int NW> struct BandShape {
+    static constexpr int LPX = 4 * NW;           // pixels per lane
+    static constexpr int STRIP = 32 * LPX;       // columns per warp
+    static constexpr int SLOT = 32 + STRIP;      // [12,16) left halo word, [16,16+STRIP) strip, then right
+    static constexpr int MINB = NW == 2 ? 8 : 5; // resident CTAs per SM (register cap)
+};
+
+struct BandGeom {
+    int w, h, pitch, out_pitch, mode;
+    int nstrip, ngx, nband;  // strips, CTA columns, bands
+    int sx0, sx1, by0, by1;  // Body strips [sx0, sx1), Body bands [by0, by1)
+};
+
+struct LapBandParams {
+    BandGeom g;
+    const uint8_t *img;
+    uint8_t *out;
+    uint32_t cword;  // the constant in all four bytes
+};
+
+__device__ __forceinline__ uint32_t su32(const void *p) { return (uint32_t)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void cpa_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cpa_wait()
+{
+    asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory");
+}
+
+__device__ __forceinline__ void band_rows(int b, int nb, int h, int &y0, int &y1)
+{
+    y0 = (int)((long long)b * h / nb);
+    y1 = (int)((long long)(b + 1) * h / nb);
+}
+
+// Row y through the border pattern for an overshoot of at most the window's
+// reach (one reflection: the launch requires h >= 8); -1: Constant, row outside.
+template <bool CHK>
+__device__ __forceinline__ int map_row1(int y, int h, int mode)
+{
+    if (!CHK || (y >= 0 && y < h)) return y;
+    switch (mode) {
+    case ISP_CLAMP: return y < 0 ? 0 : h - 1;
+    case ISP_MIRROR: return y < 0 ? -y - 1 : 2 * h - 1 - y;
+    case ISP_REPEAT: return y < 0 ? y + h : y - h;
+    default: return -1;
+    }
+}
+
+// cp.async of the lane's NW words, predicated on the lane (lanes past the image copy
+// nothing, so the halo words stored in their positions survive)
+template <int NW>
+__device__ __forceinline__ void cpa_own(uint32_t dst, const void *src, uint32_t on)
+{
+    if constexpr (NW == 4)
+        asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %2, 0;\n\t@q cp.async.cg.shared.global [%0], [%1], 16;\n\t}" ::"r"(dst),
+                     "l"(src), "r"(on)
+                     : "memory");
+    else
+        asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %2, 0;\n\t@q cp.async.ca.shared.global [%0], [%1], 8;\n\t}" ::"r"(dst),
+                     "l"(src), "r"(on)
+                     : "memory");
+}
+// 4-byte cp.async issued only by the lanes with `on` set (a predicated LDGSTS: the other
+// lanes take no part, so the instruction costs one lane of shared-memory traffic)
+__device__ __forceinline__ void cpa4p(uint32_t dst, const void *src, uint32_t on)
+{
+    asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %2, 0;\n\t@q cp.async.ca.shared.global [%0], [%1], 4;\n\t}" ::"r"(dst),
+                 "l"(src), "r"(on)
+                 : "memory");
+}
+__device__ __forceinline__ uint32_t lds32(uint32_t a)
+{
+    uint32_t v;
+    asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(a) : "memory");
+    return v;
+}
+template <int NW>
+__device__ __forceinline__ void lds_own(uint32_t a, uint32_t (&w)[NW])
+{
+    if constexpr (NW == 4)
+        asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(w[0]), "=r"(w[1]), "=r"(w[2]), "=r"(w[3]) : "r"(a)
+                     : "memory");
+    else
+        asm volatile("ld.shared.v2.u32 {%0, %1}, [%2];" : "=r"(w[0]), "=r"(w[1]) : "r"(a) : "memory");
+}
+__device__ __forceinline__ void sts32(uint32_t a, uint32_t v)
+{
+    asm volatile("st.shared.u32 [%0], %1;" ::"r"(a), "r"(v) : "memory");
+}
+// 16-bit pair lanes of a word: (b0, b2) and (b1, b3)
+__device__ __forceinline__ uint32_t ev(uint32_t w) { return __byte_perm(w, 0u, 0x4240); }
+__device__ __forceinline__ uint32_t od(uint32_t w) { return __byte_perm(w, 0u, 0x4341); }
+
+// One warp's band: input rows y0-2 .. y0+rows+1 streamed through the warp's ring (shared
+// address `ring`, LR slots), LD rows in flight.  Region handling (Listing 3 per warp):
+//   * T / B (CY): rows outside the image are mapped through the pattern when they are
+//     copied, once per row (Constant: the staged row is C);
+//   * L / R (cl / cr): only the edge lanes' halo words differ -- the wrapped word is copied
+//     (Repeat), the constant pre-stored (Constant), or the word is rebuilt from the lane's
+//     own edge bytes by a byte permute chosen once per warp (Clamp / Mirror; every other
+//     lane's selector is the identity), so the row loop itself carries no checks at all.
+template <int NW, bool CY>
+__device__ __forceinline__ void lap_band_body(const LapBandParams &p, uint32_t ring, int xs0, int y0, int rows,
+                                              int lane, bool cl, bool cr)
+{
+    using B = BandShape<NW>;
+    constexpr int LPX = B::LPX, STRIP = B::STRIP, SLOT = B::SLOT;
+    const BandGeom &g = p.g;
+    const int x = xs0 + LPX * lane;
+    const bool active = !cr || x < g.w;
+    const bool redge = cr && x + LPX == g.w;   // the image's last lane (R region)
+    const int nin = rows + 4;                  // >= 10 (bands of >= 6 rows)
+    const uint32_t loff = LPX * lane;
+    // copies per row: the lane's NW words (none past the image) and two predicated
+    // 4-byte halo copies -- A: lane 0, the strip's left word (L, Repeat: the wrapped word
+    // w-4..w-1); B: lane 31 the strip's right word, or (R, Repeat) the last lane the
+    // wrapped word 0..3 into its right neighbour's position
+    int acol = xs0 - 4, bcol = xs0 + STRIP;
+    uint32_t aon = lane == 0 && (!cl || g.mode == ISP_REPEAT), bdst = 16 + STRIP, bon = !cr && lane == 31;
+    if (cl) acol = g.w - 4;
+    if (redge && g.mode == ISP_REPEAT) { bon = 1; bcol = 0; bdst = 16 + LPX * (lane + 1); }
+    // halo selectors: W[0] = prmt(W[0], W[1], sl_), W[NW+1] = prmt(W[NW+1], W[NW], sr_)
+    uint32_t sl_ = 0x3210, sr_ = 0x3210;
+    if (cl && lane == 0) sl_ = g.mode == ISP_CLAMP ? 0x4444 : g.mode == ISP_MIRROR ? 0x4500 : 0x3210;
+    if (redge) sr_ = g.mode == ISP_CLAMP ? 0x7777 : g.mode == ISP_MIRROR ? 0x0067 : 0x3210;
+    if (g.mode == ISP_CONSTANT) {   // the halo positions no copy writes hold C in every slot
+        for (int j = 0; j < LR; ++j) {
+            if (cl && lane == 0) sts32(ring + j * SLOT + 12, p.cword);
+            if (redge) sts32(ring + j * SLOT + 16 + LPX * (lane + 1), p.cword);
+        }
+    }
+    const int mcol = active ? x : 0;
+    const uint8_t *nrp = p.img + (ptrdiff_t)(y0 - 2) * g.pitch;   // next row to issue (unmapped)
+    auto issue = [&](int j, uint32_t slot) {
+        const uint8_t *rp = nrp;
+        if constexpr (CY) {   // T / B regions: the row through the pattern, once per row
+            const int yy = map_row1<true>(y0 - 2 + j, g.h, g.mode);
+            if (yy < 0) {     // Constant: the whole staged row is C
+#pragma unroll
+                for (int q = 0; q < NW; ++q) sts32(slot + 16 + loff + 4 * q, p.cword);
+                if (lane == 0) sts32(slot + 12, p.cword);
+                if (lane == 31) sts32(slot + 16 + STRIP, p.cword);
+                return;
+            }
+            rp = p.img + (size_t)yy * g.pitch;
+        }
+        cpa_own<NW>(slot + 16 + loff, rp + mcol, active);
+        cpa4p(slot + 12, rp + acol, aon);
+        cpa4p(slot + bdst, rp + bcol, bon);
+    };
+#pragma unroll
+    for (int j = 0; j < LD; ++j) {
+        issue(j, ring + j * SLOT);
+        nrp += g.pitch;
+        cpa_commit();
+    }
+    // H ring: horizontal 5-sums of the last five rows as pair lanes, per 4-pixel group g
+    // (E_g, O_g) = ((H_4g, H_4g+2), (H_4g+1, H_4g+3)); box = sum of the ring + bias 6400
+    uint32_t hr[5][2 * NW] = {};
+    uint32_t box[2 * NW];
+#pragma unroll
+    for (int q = 0; q < 2 * NW; ++q) box[q] = 0x19001900u;
+    uint32_t c1[NW] = {}, c2[NW] = {};   // own words of rows i-1, i-2 (the centre row)
+    uint8_t *orow = p.out + (size_t)y0 * g.out_pitch + x;
+#pragma unroll 1
+    for (int i0 = 0; i0 < nin; i0 += 5) {
+#pragma unroll
+        for (int k = 0; k < 5; ++k) {
+            const int i = i0 + k;
+            if (i < nin) {
+                cpa_wait<LD - 1>();
+                __syncwarp();
+                const uint32_t sl = ring + (i & (LR - 1)) * SLOT + loff;
+                uint32_t W[NW + 2];   // W[0] = left halo word, W[1..NW] own, W[NW+1] right
+                lds_own<NW>(sl + 16, *reinterpret_cast<uint32_t(*)[NW]>(&W[1]));
+                W[0] = __byte_perm(lds32(sl + 12), W[1], sl_);
+                W[NW + 1] = __byte_perm(lds32(sl + 16 + LPX), W[NW], sr_);
+                // horizontal 5-sums on pair lanes: E_k = (b_k, b_k+2), O_k = (b_k+1, b_k+3);
+                // group g (pixels 4g..4g+3): (H,H+2) = S + E_-2, (H+1,H+3) = S + O_2 with
+                // S = O_-2 + E_0 + O_0 + E_2 (offsets relative to 4g); F_g = bytes 4g-2..4g+1
+                uint32_t Ef[NW + 1], Of[NW + 1];
+#pragma unroll
+                for (int q = 0; q <= NW; ++q) {
+                    const uint32_t F = __funnelshift_r(W[q], W[q + 1], 16);
+                    Ef[q] = ev(F);
+                    Of[q] = od(F);
+                }
+                uint32_t hn[2 * NW];
+#pragma unroll
+                for (int q = 0; q < NW; ++q) {
+                    const uint32_t S = Of[q] + ev(W[q + 1]) + od(W[q + 1]) + Ef[q + 1];
+                    hn[2 * q] = S + Ef[q];
+                    hn[2 * q + 1] = S + Of[q + 1];
+                }
+                // box of rows i-4..i: + H(i) - H(i-5) (the ring slot being replaced; zero
+                // for i < 5)
+#pragma unroll
+                for (int q = 0; q < 2 * NW; ++q) {
+                    box[q] = box[q] + hn[q] - hr[k][q];
+                    hr[k][q] = hn[q];
+                }
+                if (i >= 4) {
+                    // output row y0 + i - 4: clamp(box - 25 c, 0, 255), c = row i - 2
+                    uint32_t o[NW];
+#pragma unroll
+                    for (int q = 0; q < NW; ++q) {
+                        uint32_t vE = box[2 * q] - 25u * ev(c2[q]), vO = box[2 * q + 1] - 25u * od(c2[q]);
+                        asm("max.u16x2 %0, %0, %1;" : "+r"(vE) : "r"(0x19001900u));
+                        asm("min.u16x2 %0, %0, %1;" : "+r"(vE) : "r"(0x19FF19FFu));
+                        asm("max.u16x2 %0, %0, %1;" : "+r"(vO) : "r"(0x19001900u));
+                        asm("min.u16x2 %0, %0, %1;" : "+r"(vO) : "r"(0x19FF19FFu));
+                        o[q] = __byte_perm(vE, vO, 0x6240);
+                    }
+                    if (active) {
+                        if constexpr (NW == 4) *reinterpret_cast<uint4 *>(orow) = make_uint4(o[0], o[1], o[2], o[3]);
+                        else *reinterpret_cast<uint2 *>(orow) = make_uint2(o[0], o[1]);
+                    }
+                    orow += g.out_pitch;
+                }
+#pragma unroll
+                for (int q = 0; q < NW; ++q) {
+                    c2[q] = c1[q];
+                    c1[q] = W[q + 1];
+                }
+                // refill: row i + LD into the slot of row i + LD - LR (last read at i - 1)
+                if (i + LD < nin) issue(i + LD, ring + ((i + LD) & (LR - 1)) * SLOT);
+                nrp += g.pitch;
+                cpa_commit();
+            }
+        }
+    }
+}
+
+template <int NW>
+__global__ void __launch_bounds__(NTB, BandShape<NW>::MINB) k_lap_band(const __grid_constant__ LapBandParams p)
+{
+    using B = BandShape<NW>;
+    __shared__ __align__(16) uint8_t rings[BW][LR * B::SLOT];
+    asm volatile("griddepcontrol.wait;" ::: "memory");
+    asm volatile("griddepcontrol.launch_dependents;");
+    const BandGeom &g = p.g;
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int gx = (int)blockIdx.x % g.ngx, band = (int)blockIdx.x / g.ngx;
+    const int s = gx * BW + warp;
+    if (s >= g.nstrip) return;
+    int y0, y1;
+    band_rows(band, g.nband, g.h, y0, y1);
+    const int xs0 = s * B::STRIP;
+    // region of this warp (Listing 3 on strip / band indices, warp-uniform): T / B warps run
+    // the row-mapping body, L / R warps set their edge lanes' halo handling
+    const bool cl = s < g.sx0, cr = s >= g.sx1, cy = band < g.by0 || band >= g.by1;
+    const uint32_t ring = su32(rings[warp]);
+    if (cy) lap_band_body<NW, true>(p, ring, xs0, y0, y1 - y0, lane, cl, cr);
+    else lap_band_body<NW, false>(p, ring, xs0, y0, y1 - y0, lane, cl, cr);
+}
+
+int num_sms()
+{
+    static int n = 0;
+    if (n == 0) {
+        int dev = 0;
+        if (cudaGetDevice(&dev) != cudaSuccess || cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev) !=
+                                                      cudaSuccess) {
+            cudaGetLastError();
+            n = 148;
+        }
+    }
+    return n;
+}
+
+// Words per lane of the Laplace band launch: 4 (16 pixels) unless ISP_BAND_NW=2
+int band_nw()
+{
+    const char *e = getenv("ISP_BAND_NW");
+    return e && atoi(e) == 2 ? 2 : 4;
+}
+
+const void *lap_band_fn(int nw) { return nw == 2 ? (const void *)k_lap_band<2> : (const void *)k_lap_band<4>; }
+
+int lap_band_blocks_per_sm(int nw)
+{
+    static int nb[5] = {-1, -1, -1, -1, -1};
+    if (nb[nw] < 0) {
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb[nw], lap_band_fn(nw), NTB, 0) != cudaSuccess) {
+            cudaGetLastError();
+            nb[nw] = 0;
+        }
+    }
+    return nb[nw];
+}
+
+// Strips, bands and the Body rectangle (hy rows of reach; a strip's right halo word lies
+// past it, so a strip is Body iff it ends before the image's last column).
+BandGeom band_geom(int w, int h, int pitch, int out_pitch, int mode, int hy, int nw, int bands_hint)
+{
+    const int strip = 128 * nw;
+    BandGeom g{};
+    g.w = w; g.h = h; g.pitch = pitch; g.out_pitch = out_pitch; g.mode = mode;
+    g.nstrip = (w + strip - 1) / strip;
+    g.ngx = (g.nstrip + BW - 1) / BW;
+    int nb = bands_hint;
+    if (nb <= 0) {
+        const int per_sm = std::max(1, lap_band_blocks_per_sm(nw));
+        nb = std::max(1, num_sms() * per_sm / g.ngx);
+    }
+    g.nband = std::max(1, std::min(nb, h / (2 * hy + 2)));
+    g.sx0 = 1;
+    g.sx1 = (w - 1) / strip;
+    g.by0 = g.nband;
+    g.by1 = g.nband;
+    for (int b = g.nband - 1; b >= 0; --b) {
+        const int y0 = (int)((long long)b * h / g.nband), y1 = (int)((long long)(b + 1) * h / g.nband);
+        if (y0 >= hy) g.by0 = b;
+        if (y1 + hy > h) g.by1 = b;
+    }
+    if (g.by1 < g.by0) g.by1 = g.by0;
+    return g;
+}
+
+cudaError_t launch_band(const void *fn, void *params, int nblocks, cudaStream_t st)
+{
+    cudaLaunchConfig_t cfg{};
+    cfg.gridDim = dim3(nblocks);
+    cfg.blockDim = dim3(NTB);
+    cfg.stream = st;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    at[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    void *args[] = {params};
+    return cudaLaunchKernelExC(&cfg, fn, args);
+}
+
+int bands_hint()
+{
+    const char *e = getenv("ISP_BAND_BANDS");
+    return e ? atoi(e) : 0;
+}
+
+}  // namespace
+
+// Eligibility of the band kernels: 16-pixel lane granules (w % 16 == 0; 8 with
+// ISP_BAND_NW=2), rows aligned to the granule in and out (cp.async / vector stores), and
+// h >= 8 so that every overshoot needs one reflection.
+bool ispi_band_ok(const void *in, int w, int h, int pitch, const void *out, int out_pitch)
+{
+    const int v = 4 * band_nw();
+    auto al = [](const void *q, long long pb, int a) { return q && ((uintptr_t)q % a) == 0 && (pb % a) == 0; };
+    return al(in, pitch, v) && al(out, out_pitch, v) && w % v == 0 && w >= 2 * v && h >= 8;
+}
+
+// Strip width and band height of the Laplace band launch (the model's tile shape, Eq. 2 / 10).
+void ispi_band_shape(int w, int h, int *tw, int *th)
+{
+    const int nw = band_nw();
+    const BandGeom g = band_geom(w, h, w, w, ISP_CLAMP, 2, nw, bands_hint());
+    *tw = 128 * nw;
+    *th = (h + g.nband - 1) / g.nband;
+}
+
+int ispi_band_blocks_per_sm() { return lap_band_blocks_per_sm(band_nw()); }
+
+cudaError_t ispi_laplace_band(const uint8_t *img, int w, int h, int pitch, int mode, int cval, uint8_t *out,
+                              int out_pitch, cudaStream_t st, int bounds[4])
+{
+    const int nw = band_nw();
+    LapBandParams p{};
+    p.g = band_geom(w, h, pitch, out_pitch, mode, 2, nw, bands_hint());
+    p.img = img;
+    p.out = out;
+    p.cword = 0x01010101u * (uint32_t)(cval & 0xff);
+    bounds[0] = p.g.sx0; bounds[1] = std::max(p.g.sx0, p.g.sx1); bounds[2] = p.g.by0; bounds[3] = p.g.by1;
+    return launch_band(lap_band_fn(nw), &p, p.g.ngx * p.g.nband, st);
+}

@@ -489,9 +489,17 @@ def test_laplace_harris_tile_kernels(isp, shape):
     d = dev(img)
     for mode in MODES:
         rlap = oracle.laplace5_u8(img, mode, 33)
-        got = host(isp.isp_laplace5_u8(d, mode, 33, variant="tma"))
+        # Laplace: a width that is not a multiple of 8 (pitch still 16-B aligned) is not
+        # band-eligible, so the tile kernel runs
+        wt = w - 4
+        got = host(isp.isp_laplace5_u8(d, mode, 33, variant="tma", w=wt))
         p = isp.isp_last_plan()
         assert p["choice"] == CODE["tma"] and p["tile_w"] == 128 and p["tile_h"] == 32, p
+        np.testing.assert_array_equal(got[:, :wt], oracle.laplace5_u8(np.ascontiguousarray(img[:, :wt]), mode, 33),
+                                      err_msg=f"laplace tile {mode}")
+        got = host(isp.isp_laplace5_u8(d, mode, 33, variant="tma"))
+        p = isp.isp_last_plan()
+        assert p["choice"] == CODE["tma"] and p["tile_w"] == 512, p   # the band kernel
         np.testing.assert_array_equal(got, rlap, err_msg=f"laplace {mode}")
         rdx, rdy, _ = oracle.sobel(img, mode, 33)
         ddx, ddy = dev(rdx), dev(rdy)
@@ -506,3 +514,29 @@ def test_laplace_harris_tile_kernels(isp, shape):
         ry = synth.random_i16(h, w, 6)
         np.testing.assert_array_equal(host(isp.isp_harris_u8(dev(rx), dev(ry), mode, -3, 10 ** 11, variant="tma")),
                                       oracle.harris(rx, ry, mode, -3, 10 ** 11), err_msg=f"harris random {mode}")
+
+
+# ---------------------------------------------------------------- warp-strip band Laplace
+@pytest.mark.parametrize("nw", [4, 2])
+@pytest.mark.parametrize("shape", [(8, 32), (9, 48), (70, 2064), (33, 4112), (260, 528), (101, 512), (4096 // 8, 4096),
+                                   (17, 784)])
+def test_laplace_band_kernel(isp, shape, nw, monkeypatch):
+    """The warp-strip streaming Laplace (band_u8.cu) at 16 and 8 pixels per lane: strips of
+    512 / 256 columns (partial last strips down to one lane, a single strip that is both L
+    and R), bands down to 6 rows (T and B in one band), all four modes and constants 0 / 255
+    -- bit-exact against the oracle, the plan showing the band kernel ran (TMA choice,
+    strip-wide tiles)."""
+    monkeypatch.setenv("ISP_BAND_NW", str(nw))
+    h, w = shape
+    img = synth.structured_u8(h, w, 21)
+    img[0, :] = 255
+    img[:, -1] = 0
+    d = dev(img)
+    for mode in MODES:
+        for c in ((0, 255) if mode == "constant" else (0,)):
+            got = host(isp.isp_laplace5_u8(d, mode, c, variant="tma"))
+            p = isp.isp_last_plan()
+            assert p["choice"] == CODE["tma"] and p["tile_w"] == 128 * nw, p
+            np.testing.assert_array_equal(got, oracle.laplace5_u8(img, mode, c), err_msg=f"{mode} c={c}")
+    # AUTO (Eq. 10 decides between the band kernel and the naive one): still exact
+    np.testing.assert_array_equal(host(isp.isp_laplace5_u8(d, "mirror", 0)), oracle.laplace5_u8(img, "mirror", 0))

@@ -46,6 +46,8 @@ def main():
     ap.add_argument("--override", action="append", default=[""])
     ap.add_argument("--size", type=int, default=4096)
     ap.add_argument("--mode", default="mirror")
+    ap.add_argument("--env", action="append", default=[], help="KEY=VAL[,KEY=VAL] settings, one line each")
+    ap.add_argument("--only", default="", help="comma list of sobel,laplace,harris")
     a = ap.parse_args()
     n, nb = a.size, 6
     imgs = [torch.from_numpy(synth.uniform_u8(n, n, 3 + i)).cuda() for i in range(nb)]
@@ -56,7 +58,13 @@ def main():
     o3 = [torch.empty_like(i) for i in imgs]
     for i in range(nb):
         isp.isp_sobel_u8(imgs[i], a.mode, dx=dxs[i], dy=dys[i], mag=o1[i])
-    for ov in a.override:
+    settings = [("", ov) for ov in a.override] + [(e, "") for e in a.env]
+    for env, ov in settings:
+        keys = []
+        for kv in filter(None, env.split(",")):
+            k, val = kv.split("=")
+            os.environ[k] = val
+            keys.append(k)
         if ov:
             isp.isp_set_launch_override(*map(int, ov.split(",")))
         for v in a.variant or ["auto"]:
@@ -64,15 +72,20 @@ def main():
             for name, bpp, fn in [
                 ("sobel", 6, lambda i: isp.isp_sobel_u8(imgs[i % nb], a.mode, dx=dxs[i % nb], dy=dys[i % nb],
                                                         mag=o1[i % nb], variant=v)),
+                ("copy", 2, lambda i: o2[i % nb].copy_(imgs[i % nb])),   # torch copy of the same bytes
                 ("laplace", 2, lambda i: isp.isp_laplace5_u8(imgs[i % nb], a.mode, out=o2[i % nb], variant=v)),
                 ("harris", 5, lambda i: isp.isp_harris_u8(dxs[i % nb], dys[i % nb], a.mode, out=o3[i % nb], variant=v)),
             ]:
+                if a.only and name not in a.only.split(","):
+                    continue
                 us, plan = timed(fn)
                 r[name] = {"us": round(us, 2), "gbs": round(bpp * n * n / us / 1e3, 1),
                            "plan": [plan["tile_w"], plan["tile_h"], plan["nx"], plan["ny"], plan["choice"]]}
-            print(json.dumps({"variant": v, "override": ov, "px_u8": os.environ.get("ISP_LIB_PATH", ""), **r}), flush=True)
+            print(json.dumps({"variant": v, "override": ov, "env": env, "px_u8": os.environ.get("ISP_LIB_PATH", ""), **r}), flush=True)
         if ov:
             isp.isp_set_launch_override(0, 0)
+        for k in keys:
+            del os.environ[k]
 
 
 if __name__ == "__main__":
