@@ -651,22 +651,23 @@ isp_status_t resolve_and_launch(Desc &d, int fam, int w, int h, int mw, int mh, 
 // = 0) and Harris (1): ISP_TMA runs them when eligible; ISP_AUTO evaluates Eq. (10) for
 // them (form S, reading A21, calibrated constants, occupancy from the API) against the
 // naive kernel.  Returns false when the caller should take the generic path.
-// which = 2: the Laplace band kernel (band_u8.cu: warp strips of 256 columns x bands of rows)
+// which = 2 / 3: the Laplace / Harris band kernels (band_u8.cu: warp strips x bands of rows)
 bool tile_variant(int which, int fam, int mode, int w, int h, int mw, int mh, isp_variant_t v, bool ok,
                   const std::function<cudaError_t(int *)> &launch, isp_status_t &st, const char *what)
 {
     if (!(v == ISP_TMA || v == ISP_AUTO) || !ok) return false;
     int tw, th;
     if (which == 2) ispi_band_shape(w, h, &tw, &th);
+    else if (which == 3) ispi_band_harris_shape(w, h, &tw, &th);
     else ispi_tile_shape(&tw, &th);
-    Plan p = make_plan(w, h, mw / 2, mh / 2, 4, tw, th, which == 2 ? 256 : 128);
+    Plan p = make_plan(w, h, mw / 2, mh / 2, 4, tw, th, which >= 2 ? tw : 128);
     isp_plan_info info{};
     n_block(p, info.n_block);
     if (v == ISP_AUTO) {
         isp_model_params mp;
         defaults(fam, mode, mp);
         mp.form = 2;
-        const int nb = which == 2 ? ispi_band_blocks_per_sm() : ispi_tile_blocks_per_sm(which);
+        const int nb = which >= 2 ? ispi_band_blocks_per_sm(which == 3 ? 1 : 0) : ispi_tile_blocks_per_sm(which);
         info.o_isp = occupancy_of(nb > 0 ? nb : 1, 128);
         info.o_naive = 0.5;   // the naive streaming kernel (64 regs x 128 threads: 8 blocks / SM)
         model(p, w, h, mw, mh, mp, info);
@@ -678,7 +679,7 @@ bool tile_variant(int which, int fam, int mode, int w, int h, int mw, int mh, is
     info.bh_l = b[0]; info.bh_r = b[1]; info.bh_t = b[2]; info.bh_b = b[3];
     info.nx = p.nx; info.ny = p.ny;
     info.degenerate = 0;
-    info.tile_w = tw; info.tile_h = th; info.warp_w = which == 2 ? 256 : 128;
+    info.tile_w = tw; info.tile_h = th; info.warp_w = which >= 2 ? tw : 128;
     info.choice = ISP_TMA;
     g_last_plan = info;
     g_recent[g_n_plans++ % kRecent] = info;
@@ -1145,6 +1146,13 @@ isp_status_t isp_harris_u8(const int16_t *dx, const int16_t *dy, int w, int h, i
     if (ranges_overlap(dx, img_bytes(w, h, pitch, 2), out, ob) || ranges_overlap(dy, img_bytes(w, h, pitch, 2), out, ob))
         return fail(ISP_EALIAS, "input and output overlap");
     isp_status_t ts;
+    // ISP_TMA / AUTO: the band kernel (band_u8.cu) when eligible, else the tile kernel
+    if (tile_variant(3, F_HARRIS, border_mode, w, h, 3, 3, variant,
+                     ispi_band_harris_ok(dx, dy, w, h, pitch, out, out_pitch),
+                     [&](int *b) { return ispi_harris_band(dx, dy, w, h, pitch, border_mode, const_val, thr, out,
+                                                           out_pitch, (cudaStream_t)stream, b); },
+                     ts, "isp_harris_u8(band)"))
+        return ts;
     if (tile_variant(1, F_HARRIS, border_mode, w, h, 3, 3, variant, ispi_tile_ok(dx, dy, 2, w, h, pitch, out, out_pitch),
                      [&](int *b) { return ispi_harris_tile(dx, dy, w, h, pitch, border_mode, const_val, thr, out,
                                                            out_pitch, (cudaStream_t)stream, b); },

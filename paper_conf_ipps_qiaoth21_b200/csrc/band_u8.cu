@@ -1,5 +1,5 @@
 // band_u8.cu -- warp-strip streaming ISP kernels for the cfg3 u8 operators (round 3): the
-// ISP_TMA variant of isp_laplace5_u8 (a8).
+// ISP_TMA variant of isp_laplace5_u8 (a8) and isp_harris_u8 (a10).
 //
 // Partition (Listing 3, at warp granularity as in Listing 5): the
 // image is cut into vertical strips of 32 lanes x 4*NW pixels (one warp each; NW = 2 or 4 words) and horizontal
@@ -26,10 +26,12 @@
 #include <stdint.h>
 
 #include <algorithm>
+#include <cmath>
 #include <cstdlib>
 
 #include "../../include/isp.h"
 #include "internal.h"
+#include "harris_core.cuh"
 
 namespace {
 
@@ -299,6 +301,222 @@ __global__ void __launch_bounds__(NTB, BandShape<NW>::MINB) k_lap_band(const __g
     else lap_band_body<NW, false>(p, ring, xs0, y0, y1 - y0, lane, cl, cr);
 }
 
+
+// ------------------------------------------------------------------------------ Harris
+// Same skeleton over the int16 derivative images (a10): 4 pixels per lane (one 8-byte word
+// pair per image), strips of 128 columns, the ring slot holding the dx row then the dy row
+// (each with its two halo words), rows y0-1 .. y0+rows.  Per row the lane forms the
+// horizontal [1,2,1] sums of dx^2, dy^2, dx*dy as exact FP32x2 pairs (E = pixels (0,2),
+// O = (1,3)), keeps the last three in a register ring and decides R25 > thr exactly
+// (harris_core.cuh).  Border handling as in the Laplace body: rows mapped at copy time,
+// the edge lanes' halo words by per-warp selectors (Constant: C pre-stored).
+struct HarBandParams {
+    BandGeom g;
+    const int16_t *dx, *dy;
+    uint8_t *out;
+    uint32_t cword;   // the constant in both int16 halves
+    double thr;
+    float thr_f, thr_err;
+};
+
+constexpr int HSTRIP = 128;                 // columns per warp (4 per lane)
+constexpr int HIMG = 32 + 2 * HSTRIP;       // bytes per image row in a slot: [12,16) left, [16,272) strip, [272,276) right
+constexpr int HSLOT = 2 * HIMG;             // dx row, then dy row
+constexpr int HLD = 5;                      // rows in flight per warp
+
+struct HRow { float2 xxE, xxO, yyE, yyO, xyE, xyO; };
+
+// int16 halves of words as exact floats: w ^ 0x80008000 holds v + 32768 in each half, which
+// a byte permute places in the mantissa of 2^23 (bits 0x4B00xxxx); one packed subtract of
+// 2^23 + 32768 then yields the pair exactly.  lo: the low halves of (a, b), hi: the high.
+__device__ __forceinline__ float2 lo2(uint32_t a, uint32_t b)
+{
+    const float2 r = make_float2(__uint_as_float(__byte_perm(a ^ 0x80008000u, 0x4B000000u, 0x7610)),
+                                 __uint_as_float(__byte_perm(b ^ 0x80008000u, 0x4B000000u, 0x7610)));
+    return add2(r, f2(-8421376.0f, -8421376.0f));
+}
+__device__ __forceinline__ float2 hi2(uint32_t a, uint32_t b)
+{
+    const float2 r = make_float2(__uint_as_float(__byte_perm(a ^ 0x80008000u, 0x4B000000u, 0x7632)),
+                                 __uint_as_float(__byte_perm(b ^ 0x80008000u, 0x4B000000u, 0x7632)));
+    return add2(r, f2(-8421376.0f, -8421376.0f));
+}
+
+// Horizontal [1,2,1] sums of xx, yy, xy for pixels 0..3 from the words (L, X0, X1, R) of dx
+// and dy (L = pixels -2,-1; R = 4,5).  Products of integers <= 1020 are exact in f32.
+__device__ __forceinline__ HRow har_hrow(uint32_t XL, uint32_t X0, uint32_t X1, uint32_t XR, uint32_t YL, uint32_t Y0,
+                                         uint32_t Y1, uint32_t YR)
+{
+    const float2 xE = lo2(X0, X1), xO = hi2(X0, X1), yE = lo2(Y0, Y1), yO = hi2(Y0, Y1);
+    // edge pixels p-1 (high half of L) and p4 (low half of R) as pairs (p-1, p4)
+    const float2 xe = add2(make_float2(__uint_as_float(__byte_perm(XL ^ 0x80008000u, 0x4B000000u, 0x7632)),
+                                       __uint_as_float(__byte_perm(XR ^ 0x80008000u, 0x4B000000u, 0x7610))),
+                           f2(-8421376.0f, -8421376.0f));
+    const float2 ye = add2(make_float2(__uint_as_float(__byte_perm(YL ^ 0x80008000u, 0x4B000000u, 0x7632)),
+                                       __uint_as_float(__byte_perm(YR ^ 0x80008000u, 0x4B000000u, 0x7610))),
+                           f2(-8421376.0f, -8421376.0f));
+    const float2 xxE = mul2(xE, xE), xxO = mul2(xO, xO), yyE = mul2(yE, yE), yyO = mul2(yO, yO);
+    const float2 xyE = mul2(xE, yE), xyO = mul2(xO, yO);
+    const float2 xxe = mul2(xe, xe), yye = mul2(ye, ye), xye = mul2(xe, ye);
+    const float2 xxA = f2(xxe.x, xxO.x), xxB = f2(xxE.y, xxe.y);
+    const float2 yyA = f2(yye.x, yyO.x), yyB = f2(yyE.y, yye.y);
+    const float2 xyA = f2(xye.x, xyO.x), xyB = f2(xyE.y, xye.y);
+    const float2 two = f2(2.f, 2.f);
+    HRow h;
+    h.xxE = add2(fma2(two, xxE, xxA), xxO);   // (H0, H2) = A + 2E + O, A = (p-1, p1)
+    h.xxO = add2(fma2(two, xxO, xxE), xxB);   // (H1, H3) = E + 2O + B, B = (p2, p4)
+    h.yyE = add2(fma2(two, yyE, yyA), yyO);
+    h.yyO = add2(fma2(two, yyO, yyE), yyB);
+    h.xyE = add2(fma2(two, xyE, xyA), xyO);
+    h.xyO = add2(fma2(two, xyO, xyE), xyB);
+    return h;
+}
+
+// R25 > thr for a pixel pair, exact (reading A33).  f32 evaluation
+// R = 25 (Sxx Syy - Sxy^2) - t^2 with t = Sxx + Syy; its error is at most
+// 2^-24 (76 Sxx Syy + 51 Sxy^2 + 4.1 t^2)(1 + O(2^-24)) <= 2^-24 * 36 t^2, since
+// Sxx Syy <= t^2 / 4 (AM-GM) and Sxy^2 <= Sxx Syy (Cauchy-Schwarz, positive weights); the
+// decision bound b = 1.5 * 2^-17 * fl(t^2) + |fl(thr) - thr| (= 2^-24 * 192 t^2) covers it
+// five times over.  Pixels within the bound take the exact f64 form (t = 0: R25 = 0).
+__device__ __forceinline__ void harris2p(float2 sxx, float2 syy, float2 sxy, float thr_f, float thr_err, double thr,
+                                         uint32_t &o0, uint32_t &o1)
+{
+    const float2 pp = mul2(sxx, syy);
+    const float2 det = fma2(f2(-sxy.x, -sxy.y), sxy, pp);
+    const float2 t = add2(sxx, syy);
+    const float2 tt = mul2(t, t);
+    const float2 R = fma2(f2(25.f, 25.f), det, f2(-tt.x, -tt.y));
+    const float2 b = fma2(tt, f2(1.1444091796875e-05f, 1.1444091796875e-05f), f2(thr_err, thr_err));
+    const float2 d = add2(R, f2(-thr_f, -thr_f));
+    o0 = d.x > b.x ? 255u : 0u;
+    o1 = d.y > b.y ? 255u : 0u;
+    const bool u0 = fabsf(d.x) <= b.x, u1 = fabsf(d.y) <= b.y;   // undecided by the bound
+    if (__any_sync(0xffffffffu, u0 || u1)) {
+        if (u0) o0 = tt.x == 0.f ? (0.0 > thr ? 255u : 0u) : (uint32_t)harris_exact(sxx.x, syy.x, sxy.x, thr);
+        if (u1) o1 = tt.y == 0.f ? (0.0 > thr ? 255u : 0u) : (uint32_t)harris_exact(sxx.y, syy.y, sxy.y, thr);
+    }
+}
+
+template <bool CY>
+__device__ __forceinline__ void har_band_body(const HarBandParams &p, uint32_t ring, int xs0, int y0, int rows,
+                                              int lane, bool cl, bool cr)
+{
+    const BandGeom &g = p.g;
+    const int x = xs0 + 4 * lane;
+    const bool active = !cr || x < g.w;
+    const bool redge = cr && x + 4 == g.w;
+    const int nin = rows + 2;   // >= 8
+    const uint32_t loff = 8 * lane;
+    // halo copies (columns, in int16 elements): A = lane 0's left word (L, Repeat: w-2, w-1),
+    // B = lane 31's right word, or (R, Repeat) the last lane's wrapped word (0, 1)
+    int acol = xs0 - 2, bcol = xs0 + HSTRIP;
+    uint32_t aon = lane == 0 && (!cl || g.mode == ISP_REPEAT), bdst = 16 + 2 * HSTRIP, bon = !cr && lane == 31;
+    if (cl) acol = g.w - 2;
+    if (redge && g.mode == ISP_REPEAT) { bon = 1; bcol = 0; bdst = 16 + 8 * (lane + 1); }
+    // selectors: left word = prmt(loaded, own X0, sl_), right = prmt(loaded, own X1, sr_)
+    uint32_t sl_ = 0x3210, sr_ = 0x3210;
+    if (cl && lane == 0) sl_ = g.mode == ISP_CLAMP ? 0x5454 : g.mode == ISP_MIRROR ? 0x5476 : 0x3210;
+    if (redge) sr_ = g.mode == ISP_CLAMP ? 0x7676 : g.mode == ISP_MIRROR ? 0x5476 : 0x3210;
+    if (g.mode == ISP_CONSTANT) {
+        for (int j = 0; j < LR; ++j)
+            for (int im = 0; im < 2; ++im) {
+                if (cl && lane == 0) sts32(ring + j * HSLOT + im * HIMG + 12, p.cword);
+                if (redge) sts32(ring + j * HSLOT + im * HIMG + 16 + 8 * (lane + 1), p.cword);
+            }
+    }
+    const int mcol = active ? x : 0;
+    const size_t pitchb = (size_t)g.pitch * 2;
+    const char *nx = reinterpret_cast<const char *>(p.dx) + (ptrdiff_t)(y0 - 1) * (ptrdiff_t)pitchb;
+    const char *ny = reinterpret_cast<const char *>(p.dy) + (ptrdiff_t)(y0 - 1) * (ptrdiff_t)pitchb;
+    auto issue = [&](int j, uint32_t slot) {
+        const char *rx = nx, *ry = ny;
+        if constexpr (CY) {
+            const int yy = map_row1<true>(y0 - 1 + j, g.h, g.mode);
+            if (yy < 0) {   // Constant: both staged rows are C
+                for (int im = 0; im < 2; ++im) {
+                    sts32(slot + im * HIMG + 16 + loff, p.cword);
+                    sts32(slot + im * HIMG + 20 + loff, p.cword);
+                    if (lane == 0) sts32(slot + im * HIMG + 12, p.cword);
+                    if (lane == 31) sts32(slot + im * HIMG + 16 + 2 * HSTRIP, p.cword);
+                }
+                return;
+            }
+            rx = reinterpret_cast<const char *>(p.dx) + (size_t)yy * pitchb;
+            ry = reinterpret_cast<const char *>(p.dy) + (size_t)yy * pitchb;
+        }
+        cpa_own<2>(slot + 16 + loff, rx + 2 * mcol, active);
+        cpa_own<2>(slot + HIMG + 16 + loff, ry + 2 * mcol, active);
+        cpa4p(slot + 12, rx + 2 * acol, aon);
+        cpa4p(slot + HIMG + 12, ry + 2 * acol, aon);
+        cpa4p(slot + bdst, rx + 2 * bcol, bon);
+        cpa4p(slot + HIMG + bdst, ry + 2 * bcol, bon);
+    };
+#pragma unroll
+    for (int j = 0; j < HLD; ++j) {
+        issue(j, ring + j * HSLOT);
+        nx += pitchb;
+        ny += pitchb;
+        cpa_commit();
+    }
+    HRow hr[3];
+    uint8_t *orow = p.out + (size_t)y0 * g.out_pitch + x;
+    const float2 two = f2(2.f, 2.f);
+#pragma unroll 1
+    for (int i0 = 0; i0 < nin; i0 += 3) {
+#pragma unroll
+        for (int k = 0; k < 3; ++k) {
+            const int i = i0 + k;
+            if (i < nin) {
+                cpa_wait<HLD - 1>();
+                __syncwarp();
+                const uint32_t sl = ring + (i & (LR - 1)) * HSLOT + loff;
+                uint32_t X[2], Y[2];
+                lds_own<2>(sl + 16, X);
+                lds_own<2>(sl + HIMG + 16, Y);
+                const uint32_t XL = __byte_perm(lds32(sl + 12), X[0], sl_), YL = __byte_perm(lds32(sl + HIMG + 12), Y[0], sl_);
+                const uint32_t XR = __byte_perm(lds32(sl + 24), X[1], sr_), YR = __byte_perm(lds32(sl + HIMG + 24), Y[1], sr_);
+                hr[k] = har_hrow(XL, X[0], X[1], XR, YL, Y[0], Y[1], YR);
+                if (i >= 2) {
+                    // output row y0 + i - 2: rows i-2, i-1, i are hr[k+1], hr[k+2], hr[k] (mod 3)
+                    const HRow &a = hr[(k + 1) % 3], &b = hr[(k + 2) % 3], &c = hr[k];
+                    const float2 sxxE = add2(fma2(two, b.xxE, a.xxE), c.xxE), sxxO = add2(fma2(two, b.xxO, a.xxO), c.xxO);
+                    const float2 syyE = add2(fma2(two, b.yyE, a.yyE), c.yyE), syyO = add2(fma2(two, b.yyO, a.yyO), c.yyO);
+                    const float2 sxyE = add2(fma2(two, b.xyE, a.xyE), c.xyE), sxyO = add2(fma2(two, b.xyO, a.xyO), c.xyO);
+                    uint32_t h0, h1, h2, h3;
+                    harris2p(sxxE, syyE, sxyE, p.thr_f, p.thr_err, p.thr, h0, h2);
+                    harris2p(sxxO, syyO, sxyO, p.thr_f, p.thr_err, p.thr, h1, h3);
+                    if (active)   // bytes (h0, h1, h2, h3)
+                        *reinterpret_cast<uint32_t *>(orow) =
+                            __byte_perm(__byte_perm(h0, h1, 0x0040), __byte_perm(h2, h3, 0x0040), 0x5410);
+                    orow += g.out_pitch;
+                }
+                if (i + HLD < nin) issue(i + HLD, ring + ((i + HLD) & (LR - 1)) * HSLOT);
+                nx += pitchb;
+                ny += pitchb;
+                cpa_commit();
+            }
+        }
+    }
+}
+
+__global__ void __launch_bounds__(NTB, 4) k_har_band(const __grid_constant__ HarBandParams p)
+{
+    __shared__ __align__(16) uint8_t rings[BW][LR * HSLOT];
+    asm volatile("griddepcontrol.wait;" ::: "memory");
+    asm volatile("griddepcontrol.launch_dependents;");
+    const BandGeom &g = p.g;
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int gx = (int)blockIdx.x % g.ngx, band = (int)blockIdx.x / g.ngx;
+    const int s = gx * BW + warp;
+    if (s >= g.nstrip) return;
+    int y0, y1;
+    band_rows(band, g.nband, g.h, y0, y1);
+    const bool cl = s < g.sx0, cr = s >= g.sx1, cy = band < g.by0 || band >= g.by1;
+    const uint32_t ring = su32(rings[warp]);
+    if (cy) har_band_body<true>(p, ring, s * HSTRIP, y0, y1 - y0, lane, cl, cr);
+    else har_band_body<false>(p, ring, s * HSTRIP, y0, y1 - y0, lane, cl, cr);
+}
+
 int num_sms()
 {
     static int n = 0;
@@ -322,31 +540,31 @@ int band_nw()
 
 const void *lap_band_fn(int nw) { return nw == 2 ? (const void *)k_lap_band<2> : (const void *)k_lap_band<4>; }
 
-int lap_band_blocks_per_sm(int nw)
+// resident CTAs per SM: which = 2 / 4 (Laplace, NW words per lane), 1 (Harris)
+int band_blocks_per_sm(int which)
 {
     static int nb[5] = {-1, -1, -1, -1, -1};
-    if (nb[nw] < 0) {
-        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb[nw], lap_band_fn(nw), NTB, 0) != cudaSuccess) {
+    if (nb[which] < 0) {
+        const void *fn = which == 1 ? (const void *)k_har_band : lap_band_fn(which);
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb[which], fn, NTB, 0) != cudaSuccess) {
             cudaGetLastError();
-            nb[nw] = 0;
+            nb[which] = 0;
         }
     }
-    return nb[nw];
+    return nb[which];
 }
 
 // Strips, bands and the Body rectangle (hy rows of reach; a strip's right halo word lies
 // past it, so a strip is Body iff it ends before the image's last column).
-BandGeom band_geom(int w, int h, int pitch, int out_pitch, int mode, int hy, int nw, int bands_hint)
+BandGeom band_geom(int w, int h, int pitch, int out_pitch, int mode, int hy, int strip, int per_sm, int bands_hint)
 {
-    const int strip = 128 * nw;
     BandGeom g{};
     g.w = w; g.h = h; g.pitch = pitch; g.out_pitch = out_pitch; g.mode = mode;
     g.nstrip = (w + strip - 1) / strip;
     g.ngx = (g.nstrip + BW - 1) / BW;
     int nb = bands_hint;
     if (nb <= 0) {
-        const int per_sm = std::max(1, lap_band_blocks_per_sm(nw));
-        nb = std::max(1, num_sms() * per_sm / g.ngx);
+        nb = std::max(1, num_sms() * std::max(1, per_sm) / g.ngx);
     }
     g.nband = std::max(1, std::min(nb, h / (2 * hy + 2)));
     g.sx0 = 1;
@@ -399,22 +617,53 @@ bool ispi_band_ok(const void *in, int w, int h, int pitch, const void *out, int 
 void ispi_band_shape(int w, int h, int *tw, int *th)
 {
     const int nw = band_nw();
-    const BandGeom g = band_geom(w, h, w, w, ISP_CLAMP, 2, nw, bands_hint());
+    const BandGeom g = band_geom(w, h, w, w, ISP_CLAMP, 2, 128 * nw, band_blocks_per_sm(nw), bands_hint());
     *tw = 128 * nw;
     *th = (h + g.nband - 1) / g.nband;
 }
 
-int ispi_band_blocks_per_sm() { return lap_band_blocks_per_sm(band_nw()); }
+int ispi_band_blocks_per_sm(int which) { return band_blocks_per_sm(which == 1 ? 1 : band_nw()); }
 
 cudaError_t ispi_laplace_band(const uint8_t *img, int w, int h, int pitch, int mode, int cval, uint8_t *out,
                               int out_pitch, cudaStream_t st, int bounds[4])
 {
     const int nw = band_nw();
     LapBandParams p{};
-    p.g = band_geom(w, h, pitch, out_pitch, mode, 2, nw, bands_hint());
+    p.g = band_geom(w, h, pitch, out_pitch, mode, 2, 128 * nw, band_blocks_per_sm(nw), bands_hint());
     p.img = img;
     p.out = out;
     p.cword = 0x01010101u * (uint32_t)(cval & 0xff);
     bounds[0] = p.g.sx0; bounds[1] = std::max(p.g.sx0, p.g.sx1); bounds[2] = p.g.by0; bounds[3] = p.g.by1;
     return launch_band(lap_band_fn(nw), &p, p.g.ngx * p.g.nband, st);
+}
+
+// Harris band kernel: 4-pixel lane granules of int16 (8-byte aligned rows), 4-byte aligned
+// output rows, h >= 8.
+bool ispi_band_harris_ok(const void *dx, const void *dy, int w, int h, int pitch, const void *out, int out_pitch)
+{
+    auto al = [](const void *q, long long pb, int a) { return q && ((uintptr_t)q % a) == 0 && (pb % a) == 0; };
+    return al(dx, 2LL * pitch, 8) && al(dy, 2LL * pitch, 8) && al(out, out_pitch, 4) && w % 4 == 0 && w >= 8 && h >= 8;
+}
+
+void ispi_band_harris_shape(int w, int h, int *tw, int *th)
+{
+    const BandGeom g = band_geom(w, h, w, w, ISP_CLAMP, 1, HSTRIP, band_blocks_per_sm(1), bands_hint());
+    *tw = HSTRIP;
+    *th = (h + g.nband - 1) / g.nband;
+}
+
+cudaError_t ispi_harris_band(const int16_t *dx, const int16_t *dy, int w, int h, int pitch, int mode, int cval,
+                             long long thr, uint8_t *out, int out_pitch, cudaStream_t st, int bounds[4])
+{
+    HarBandParams p{};
+    p.g = band_geom(w, h, pitch, out_pitch, mode, 1, HSTRIP, band_blocks_per_sm(1), bands_hint());
+    p.dx = dx;
+    p.dy = dy;
+    p.out = out;
+    p.cword = 0x00010001u * (uint32_t)(uint16_t)(int16_t)cval;
+    p.thr = (double)std::max(-9007199254740992ll, std::min(9007199254740992ll, thr));
+    p.thr_f = (float)p.thr;
+    p.thr_err = 2.0f * 5.9604645e-08f * std::fabs(p.thr_f) + 1e-30f;   // |(float)thr - thr| + margin
+    bounds[0] = p.g.sx0; bounds[1] = std::max(p.g.sx0, p.g.sx1); bounds[2] = p.g.by0; bounds[3] = p.g.by1;
+    return launch_band((const void *)k_har_band, &p, p.g.ngx * p.g.nband, st);
 }

@@ -35,9 +35,13 @@ cudaError_t ispi_laplace_tile(const uint8_t *img, int w, int h, int pitch, int m
 cudaError_t ispi_harris_tile(const int16_t *dx, const int16_t *dy, int w, int h, int pitch, int mode, int cval,
                              long long thr, uint8_t *out, int out_pitch, cudaStream_t st, int bounds[4]);
 
-// warp-strip streaming band kernels (band_u8.cu): the ISP_TMA variant of Laplace
+// warp-strip streaming band kernels (band_u8.cu): the ISP_TMA variant of Laplace and Harris
 bool ispi_band_ok(const void *in, int w, int h, int pitch, const void *out, int out_pitch);
 void ispi_band_shape(int w, int h, int *tw, int *th);
-int ispi_band_blocks_per_sm();
+int ispi_band_blocks_per_sm(int which);   // 0: Laplace, 1: Harris
+bool ispi_band_harris_ok(const void *dx, const void *dy, int w, int h, int pitch, const void *out, int out_pitch);
+void ispi_band_harris_shape(int w, int h, int *tw, int *th);
+cudaError_t ispi_harris_band(const int16_t *dx, const int16_t *dy, int w, int h, int pitch, int mode, int cval,
+                             long long thr, uint8_t *out, int out_pitch, cudaStream_t st, int bounds[4]);
 cudaError_t ispi_laplace_band(const uint8_t *img, int w, int h, int pitch, int mode, int cval, uint8_t *out,
                               int out_pitch, cudaStream_t st, int bounds[4]);

@@ -504,10 +504,20 @@ def test_laplace_harris_tile_kernels(isp, shape):
         rdx, rdy, _ = oracle.sobel(img, mode, 33)
         ddx, ddy = dev(rdx), dev(rdy)
         c = 700 if mode == "constant" else 0
+        # Harris: a width that is not a multiple of 4 runs the tile kernel, else the band one
+        wt = w - 2
+        sdx, sdy = np.ascontiguousarray(rdx[:, :wt]), np.ascontiguousarray(rdy[:, :wt])
         for thr in (0, -(10 ** 7), 10 ** 9, 10 ** 12):
+            got = host(isp.isp_harris_u8(ddx, ddy, mode, c, thr, variant="tma", w=wt,
+                                         out=torch.empty((h, w), dtype=torch.uint8, device="cuda")))
+            p = isp.isp_last_plan()
+            assert p["choice"] == CODE["tma"] and p["tile_w"] == 128 and p["tile_h"] == 32, p
+            np.testing.assert_array_equal(got[:, :wt], oracle.harris(sdx, sdy, mode, c, thr),
+                                          err_msg=f"harris tile {mode} thr={thr}")
             rhar = oracle.harris(rdx, rdy, mode, c, thr)
             got = host(isp.isp_harris_u8(ddx, ddy, mode, c, thr, variant="tma"))
-            assert isp.isp_last_plan()["choice"] == CODE["tma"]
+            p = isp.isp_last_plan()
+            assert p["choice"] == CODE["tma"] and p["tile_w"] == 128 and p["tile_h"] < 32, p   # band
             np.testing.assert_array_equal(got, rhar, err_msg=f"harris {mode} thr={thr}")
         # random int16 derivatives over the whole Sobel range
         rx = synth.random_i16(h, w, 5)
@@ -540,3 +550,27 @@ def test_laplace_band_kernel(isp, shape, nw, monkeypatch):
             np.testing.assert_array_equal(got, oracle.laplace5_u8(img, mode, c), err_msg=f"{mode} c={c}")
     # AUTO (Eq. 10 decides between the band kernel and the naive one): still exact
     np.testing.assert_array_equal(host(isp.isp_laplace5_u8(d, "mirror", 0)), oracle.laplace5_u8(img, "mirror", 0))
+
+
+@pytest.mark.parametrize("shape", [(8, 8), (9, 132), (70, 2064), (33, 4112), (101, 128), (4096 // 8, 4096), (17, 260)])
+def test_harris_band_kernel(isp, shape):
+    """The warp-strip streaming Harris (band_u8.cu): strips of 128 columns (partial last
+    strips down to one lane, one strip that is both L and R), bands down to 4 rows, all
+    modes, constants at the ends of the Sobel range, thresholds from far below to far
+    above the responses, Sobel derivatives of a structured image and random int16 over the
+    whole range -- bit-exact against the oracle's int64 definition."""
+    h, w = shape
+    img = synth.structured_u8(h, w, 23)
+    for mode in MODES:
+        rdx, rdy, _ = oracle.sobel(img, mode, 9)
+        rx = synth.random_i16(h, w, 31)
+        ry = synth.random_i16(h, w, 32)
+        for dx, dy in ((rdx, rdy), (rx, ry)):
+            ddx, ddy = dev(dx), dev(dy)
+            for c in ((-1020, 1020) if mode == "constant" else (0,)):
+                for thr in (0, -(10 ** 9), 10 ** 8, 10 ** 13):
+                    got = host(isp.isp_harris_u8(ddx, ddy, mode, c, thr, variant="tma"))
+                    p = isp.isp_last_plan()
+                    assert p["choice"] == CODE["tma"] and p["warp_w"] == 128 and p["tile_h"] < 32, p
+                    np.testing.assert_array_equal(got, oracle.harris(dx, dy, mode, c, thr),
+                                                  err_msg=f"{mode} c={c} thr={thr}")
