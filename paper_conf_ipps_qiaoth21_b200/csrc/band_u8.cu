@@ -517,6 +517,270 @@ __global__ void __launch_bounds__(NTB, 4) k_har_band(const __grid_constant__ Har
     else har_band_body<false>(p, ring, s * HSTRIP, y0, y1 - y0, lane, cl, cr);
 }
 
+
+// ------------------------------------------------------------------------------ fused cfg3
+// BASELINE configs[2] in one band launch (the ISP_TMA variant of
+// isp_pipeline_cfg3_u8): per warp a strip of 128 columns (4 pixels per lane), the u8 rows
+// y0-2 .. y0+rows+1 streamed through the cp.async ring once; per row the lane forms the
+// byte pair lanes E_k / O_k (as the Laplace body) and from them
+//   * Laplace: the horizontal 5-sum pairs, a 5-row running box (ring rotated in registers);
+//   * Sobel: horizontal parts s = a + 2b + c and d = c - a for the pairs A = (p-1, p1),
+//     E = (p0, p2), O = (p1, p3), B = (p2, p4), biased 16-bit lanes (no borrows); two rows
+//     later dx = d + 2d + d and dy = s - s (bias 1024 per lane), as exact floats;
+//   * magnitude: sqrt.approx of min(dx^2 + dy^2, 65280) rounded to nearest (DESIGN.md 7c:
+//     never within 4.9e-4 of a tie, so it equals round-half-up), read as the low byte;
+//   * Harris over the dx / dy IMAGES: horizontal [1,2,1] sums of the products (pairs A..B
+//     supply p-1 and p4), a 3-row ring, the exact decision harris2p.
+// Border handling: the image pattern for Laplace / Sobel is the staging's (rows mapped at
+// copy time, the edge lanes' halo words by selectors); Harris reads dx / dy at REMAPPED
+// coordinates, which differ from the shifted window outside the image: the edge lane of an
+// L / R warp replaces its dx / dy at column -1 / w by the value at B(-1) / B(w) (Clamp,
+// Mirror: its own column 0 / w-1; Constant: the Harris constant; Repeat: the shifted
+// window over the periodic image already is dx / dy at the wrapped column), and the band
+// holding row 0 / h-1 replaces its ext dx / dy row -1 / h likewise (row 0 / h-1, the
+// constant, or Repeat's natural value).  Bit-exact against the oracle composition.
+struct FusedBandParams {
+    BandGeom g;
+    const uint8_t *img;
+    uint8_t *mag, *lap, *har;
+    int16_t *dx, *dy;
+    uint32_t cword;     // the image constant in all four bytes
+    float c4;           // 4 hc^2: every [1,2,1] sum of a constant-hc row of products
+    float hcf;          // the Harris constant
+    double thr;
+    float thr_f, thr_err;
+};
+
+constexpr int FSTRIP = 128, FSLOT = 32 + FSTRIP, FLD = 5;
+
+struct SobH { uint32_t sA, sE, sO, sB, dA, dE, dO, dB; };
+
+// (lanes of x) - bias as floats: 2^23 + lane read from the mantissa, one packed subtract
+__device__ __forceinline__ float2 lanes_f(uint32_t x, float bias)
+{
+    const float2 r = make_float2(__uint_as_float(__byte_perm(x, 0x4B000000u, 0x7610)),
+                                 __uint_as_float(__byte_perm(x, 0x4B000000u, 0x7632)));
+    return add2(r, f2(-8388608.0f - bias, -8388608.0f - bias));
+}
+
+// Horizontal [1,2,1] sums of the products from dx / dy as the pairs A = (p-1, p1), E, O,
+// B = (p2, p4): (H0, H2) = A + 2E + O, (H1, H3) = E + 2O + B (no pair shuffling)
+__device__ __forceinline__ HRow har_hrow_f(float2 xA, float2 xE, float2 xO, float2 xB, float2 yA, float2 yE, float2 yO,
+                                           float2 yB)
+{
+    const float2 two = f2(2.f, 2.f);
+    const float2 xxE = mul2(xE, xE), xxO = mul2(xO, xO), yyE = mul2(yE, yE), yyO = mul2(yO, yO);
+    const float2 xyE = mul2(xE, yE), xyO = mul2(xO, yO);
+    HRow h;
+    h.xxE = add2(fma2(two, xxE, mul2(xA, xA)), xxO);
+    h.xxO = add2(fma2(two, xxO, xxE), mul2(xB, xB));
+    h.yyE = add2(fma2(two, yyE, mul2(yA, yA)), yyO);
+    h.yyO = add2(fma2(two, yyO, yyE), mul2(yB, yB));
+    h.xyE = add2(fma2(two, xyE, mul2(xA, yA)), xyO);
+    h.xyO = add2(fma2(two, xyO, xyE), mul2(xB, yB));
+    return h;
+}
+
+// magnitude byte of a pixel from exact float dx, dy
+__device__ __forceinline__ uint32_t mag_bits(float n)
+{
+    float r;
+    asm("sqrt.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(fminf(n, 65280.0f)));
+    return __float_as_uint(r + 8388608.0f);   // low byte = round(r) <= 255
+}
+
+template <bool CY>
+__device__ __forceinline__ void fused_band_body(const FusedBandParams &p, uint32_t ring, int xs0, int y0, int rows,
+                                                int lane, bool cl, bool cr)
+{
+    const BandGeom &g = p.g;
+    constexpr int LPX = 4;
+    const int x = xs0 + LPX * lane;
+    const bool active = !cr || x < g.w;
+    const bool redge = cr && x + LPX == g.w;
+    const int nin = rows + 4;   // >= 10
+    const uint32_t loff = LPX * lane;
+    // staging as in the Laplace body (one word per lane)
+    int acol = xs0 - 4, bcol = xs0 + FSTRIP;
+    uint32_t aon = lane == 0 && (!cl || g.mode == ISP_REPEAT), bdst = 16 + FSTRIP, bon = !cr && lane == 31;
+    if (cl) acol = g.w - 4;
+    if (redge && g.mode == ISP_REPEAT) { bon = 1; bcol = 0; bdst = 16 + LPX * (lane + 1); }
+    uint32_t sl_ = 0x3210, sr_ = 0x3210;
+    if (cl && lane == 0) sl_ = g.mode == ISP_CLAMP ? 0x4444 : g.mode == ISP_MIRROR ? 0x4500 : 0x3210;
+    if (redge) sr_ = g.mode == ISP_CLAMP ? 0x7777 : g.mode == ISP_MIRROR ? 0x0067 : 0x3210;
+    if (g.mode == ISP_CONSTANT) {
+        for (int j = 0; j < LR; ++j) {
+            if (cl && lane == 0) sts32(ring + j * FSLOT + 12, p.cword);
+            if (redge) sts32(ring + j * FSLOT + 16 + LPX * (lane + 1), p.cword);
+        }
+    }
+    // Harris' remapped dx / dy at column -1 (this lane's pixel p-1) / w (pixel p4): 1 = the
+    // lane's own column 0 / w-1 (Clamp, Mirror), 2 = the Harris constant (Constant)
+    const int rep = g.mode == ISP_REPEAT ? 0 : g.mode == ISP_CONSTANT ? 2 : 1;
+    const int ea = cl && lane == 0 ? rep : 0, eb = redge ? rep : 0;
+    const uint32_t sela = ea ? 0x3254 : 0x3210, selb = eb ? 0x7610 : 0x3210;   // low / high lane from src
+    const bool ea2 = ea == 2, eb2 = eb == 2;
+    const uint32_t hcw = 0x00010001u * (uint32_t)((int)p.hcf + 1024);             // biased constant lanes
+    // ... and at rows -1 / h: the band's first / last dx / dy row (steps 2 / nin-1) is
+    // replaced by row 0 / h-1 (copy, Clamp / Mirror) or the constant row (Constant)
+    const int fix_t = y0 == 0 && rep ? (rep == 2 ? 2 : 3) : -1;   // step of the fix
+    const int fix_b = y0 + rows == g.h && rep ? nin - 1 : -1;
+    const int mcol = active ? x : 0;
+    const uint8_t *nrp = p.img + (ptrdiff_t)(y0 - 2) * g.pitch;
+    auto issue = [&](int j, uint32_t slot) {
+        const uint8_t *rp = nrp;
+        if constexpr (CY) {
+            const int yy = map_row1<true>(y0 - 2 + j, g.h, g.mode);
+            if (yy < 0) {
+                sts32(slot + 16 + loff, p.cword);
+                if (lane == 0) sts32(slot + 12, p.cword);
+                if (lane == 31) sts32(slot + 16 + FSTRIP, p.cword);
+                return;
+            }
+            rp = p.img + (size_t)yy * g.pitch;
+        }
+        cpa4p(slot + 16 + loff, rp + mcol, active);
+        cpa4p(slot + 12, rp + acol, aon);
+        cpa4p(slot + bdst, rp + bcol, bon);
+    };
+#pragma unroll
+    for (int j = 0; j < FLD; ++j) {
+        issue(j, ring + j * FSLOT);
+        nrp += g.pitch;
+        cpa_commit();
+    }
+    // Laplace: box(i) = H(i) + Q(i-1) + Q(i-3) with Q(r) = H(r) + H(r-1), a ring of three Q
+    // by step (pairs (H0,H2), (H1,H3)), bias 6400 per lane carried by the Q ring
+    uint32_t lq[3][2] = {}, hp0 = 0, hp1 = 0;
+    SobH sr[3];                              // Sobel horizontal parts, ring by step
+    HRow hr[3];                              // Harris horizontal sums of dx / dy row (step - 2)
+    const HRow hconst = {f2(p.c4, p.c4), f2(p.c4, p.c4), f2(p.c4, p.c4), f2(p.c4, p.c4), f2(p.c4, p.c4),
+                         f2(p.c4, p.c4)};
+    const float2 two = f2(2.f, 2.f);
+    ptrdiff_t o4 = (ptrdiff_t)(y0 - 4) * g.out_pitch + x;   // output offset of row y0 + i - 4
+#pragma unroll 1
+    for (int i0 = 0; i0 < nin; i0 += 3) {
+#pragma unroll
+        for (int k = 0; k < 3; ++k) {
+            const int i = i0 + k;
+            if (i < nin) {
+                cpa_wait<FLD - 1>();
+                __syncwarp();
+                const uint32_t sl = ring + (i & (LR - 1)) * FSLOT + loff;
+                const uint32_t W0 = lds32(sl + 16);
+                const uint32_t L = __byte_perm(lds32(sl + 12), W0, sl_), R = __byte_perm(lds32(sl + 20), W0, sr_);
+                const uint32_t F0 = __funnelshift_r(L, W0, 16), F1 = __funnelshift_r(W0, R, 16);
+                const uint32_t Em2 = ev(F0), Om2 = od(F0), E0 = ev(W0), O0 = od(W0), E2 = ev(F1), O2 = od(F1);
+                // ---- Laplace (a8): box of rows i-4..i, output row y0 + i - 4
+                const uint32_t S = Om2 + E0 + O0 + E2;
+                const uint32_t hn0 = S + Em2, hn1 = S + O2;
+                const uint32_t box0 = hn0 + lq[(k + 2) % 3][0] + lq[k][0] + 0x19001900u;
+                const uint32_t box1 = hn1 + lq[(k + 2) % 3][1] + lq[k][1] + 0x19001900u;
+                lq[k][0] = hn0 + hp0;
+                lq[k][1] = hn1 + hp1;
+                hp0 = hn0;
+                hp1 = hn1;
+                // ---- Sobel horizontal parts of row i
+                SobH &sh = sr[k];
+                sh.sA = Em2 + 2u * Om2 + E0;
+                sh.sE = Om2 + 2u * E0 + O0;
+                sh.sO = E0 + 2u * O0 + E2;
+                sh.sB = O0 + 2u * E2 + O2;
+                sh.dA = E0 + 0x01000100u - Em2;
+                sh.dE = O0 + 0x01000100u - Om2;
+                sh.dO = E2 + 0x01000100u - E0;
+                sh.dB = O2 + 0x01000100u - O0;
+                if (i >= 4) {
+                    const uint32_t c2 = lds32(ring + ((i - 2) & (LR - 1)) * FSLOT + loff + 16);   // row i-2
+                    uint32_t vE = box0 - 25u * ev(c2), vO = box1 - 25u * od(c2);
+                    asm("max.u16x2 %0, %0, %1;" : "+r"(vE) : "r"(0x19001900u));
+                    asm("min.u16x2 %0, %0, %1;" : "+r"(vE) : "r"(0x19FF19FFu));
+                    asm("max.u16x2 %0, %0, %1;" : "+r"(vO) : "r"(0x19001900u));
+                    asm("min.u16x2 %0, %0, %1;" : "+r"(vO) : "r"(0x19FF19FFu));
+                    if (active) *reinterpret_cast<uint32_t *>(p.lap + o4) = __byte_perm(vE, vO, 0x6240);
+                }
+                if (i >= 2) {
+                    // ---- dx / dy of row y0 + i - 3 (rows i-2, i-1, i), as exact floats
+                    const SobH &a = sr[(k + 1) % 3], &b = sr[(k + 2) % 3];
+                    const uint32_t dxA = a.dA + 2u * b.dA + sh.dA, dxE = a.dE + 2u * b.dE + sh.dE;
+                    const uint32_t dxO = a.dO + 2u * b.dO + sh.dO, dxB = a.dB + 2u * b.dB + sh.dB;
+                    const uint32_t dyA = sh.sA + 0x04000400u - a.sA, dyE = sh.sE + 0x04000400u - a.sE;
+                    const uint32_t dyO = sh.sO + 0x04000400u - a.sO, dyB = sh.sB + 0x04000400u - a.sB;
+                    // Harris reads the dx / dy images at remapped columns (edge lanes only):
+                    // column -1 = the low lane of A, column w = the high lane of B, replaced
+                    // by a byte permute (identity elsewhere) from column 0 / w-1 or the constant
+                    const uint32_t xa = __byte_perm(dxA, ea2 ? hcw : dxE, sela), ya = __byte_perm(dyA, ea2 ? hcw : dyE, sela);
+                    const uint32_t xb = __byte_perm(dxB, eb2 ? hcw : dxO, selb), yb = __byte_perm(dyB, eb2 ? hcw : dyO, selb);
+                    const float2 xE = lanes_f(dxE, 1024.f), xO = lanes_f(dxO, 1024.f);
+                    const float2 yE = lanes_f(dyE, 1024.f), yO = lanes_f(dyO, 1024.f);
+                    const float2 xA = lanes_f(xa, 1024.f), xB = lanes_f(xb, 1024.f);
+                    const float2 yA = lanes_f(ya, 1024.f), yB = lanes_f(yb, 1024.f);
+                    hr[k] = har_hrow_f(xA, xE, xO, xB, yA, yE, yO, yB);
+                    // ... and at remapped rows (the band's first / last dx / dy row)
+                    if (i == fix_t) {
+                        if (rep == 2) hr[k] = hconst;
+                        else hr[(k + 2) % 3] = hr[k];   // step 3: row 0 also stands for row -1
+                    }
+                    if (i == fix_b) hr[k] = rep == 2 ? hconst : hr[(k + 2) % 3];
+                    // ---- magnitude (a9) and the optional dx / dy images of row y0 + i - 3
+                    if (i >= 3 && i <= rows + 2) {
+                        const ptrdiff_t o3 = o4 + g.out_pitch;
+                        const float2 nE = fma2(xE, xE, mul2(yE, yE)), nO = fma2(xO, xO, mul2(yO, yO));
+                        const uint32_t m0 = mag_bits(nE.x), m1 = mag_bits(nO.x), m2 = mag_bits(nE.y), m3 = mag_bits(nO.y);
+                        const uint32_t mw = __byte_perm(__byte_perm(m0, m1, 0x0040), __byte_perm(m2, m3, 0x0040), 0x5410);
+                        if (active) *reinterpret_cast<uint32_t *>(p.mag + o3) = mw;
+                        if (p.dx && active) {   // int16 = low half of the bits of v + 1.5 * 2^23
+                            const float2 a2 = add2(xE, f2(12582912.f, 12582912.f)), b2 = add2(xO, f2(12582912.f, 12582912.f));
+                            const float2 c2_ = add2(yE, f2(12582912.f, 12582912.f)), d2 = add2(yO, f2(12582912.f, 12582912.f));
+                            *reinterpret_cast<uint2 *>(p.dx + o3) =
+                                make_uint2(__byte_perm(__float_as_uint(a2.x), __float_as_uint(b2.x), 0x5410),
+                                           __byte_perm(__float_as_uint(a2.y), __float_as_uint(b2.y), 0x5410));
+                            *reinterpret_cast<uint2 *>(p.dy + o3) =
+                                make_uint2(__byte_perm(__float_as_uint(c2_.x), __float_as_uint(d2.x), 0x5410),
+                                           __byte_perm(__float_as_uint(c2_.y), __float_as_uint(d2.y), 0x5410));
+                        }
+                    }
+                    if (i >= 4) {
+                        // ---- Harris (a10) of row y0 + i - 4: dx / dy rows i-4 .. i-2 (steps)
+                        const HRow &ha = hr[(k + 1) % 3], &hb = hr[(k + 2) % 3], &hc = hr[k];
+                        const float2 sxxE = add2(fma2(two, hb.xxE, ha.xxE), hc.xxE), sxxO = add2(fma2(two, hb.xxO, ha.xxO), hc.xxO);
+                        const float2 syyE = add2(fma2(two, hb.yyE, ha.yyE), hc.yyE), syyO = add2(fma2(two, hb.yyO, ha.yyO), hc.yyO);
+                        const float2 sxyE = add2(fma2(two, hb.xyE, ha.xyE), hc.xyE), sxyO = add2(fma2(two, hb.xyO, ha.xyO), hc.xyO);
+                        uint32_t h0, h1, h2, h3;
+                        harris2p(sxxE, syyE, sxyE, p.thr_f, p.thr_err, p.thr, h0, h2);
+                        harris2p(sxxO, syyO, sxyO, p.thr_f, p.thr_err, p.thr, h1, h3);
+                        if (active)
+                            *reinterpret_cast<uint32_t *>(p.har + o4) =
+                                __byte_perm(__byte_perm(h0, h1, 0x0040), __byte_perm(h2, h3, 0x0040), 0x5410);
+                    }
+                }
+                o4 += g.out_pitch;
+                if (i + FLD < nin) issue(i + FLD, ring + ((i + FLD) & (LR - 1)) * FSLOT);
+                nrp += g.pitch;
+                cpa_commit();
+            }
+        }
+    }
+}
+
+__global__ void __launch_bounds__(NTB, 4) k_fused_band(const __grid_constant__ FusedBandParams p)
+{
+    __shared__ __align__(16) uint8_t rings[BW][LR * FSLOT];
+    asm volatile("griddepcontrol.wait;" ::: "memory");
+    asm volatile("griddepcontrol.launch_dependents;");
+    const BandGeom &g = p.g;
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int gx = (int)blockIdx.x % g.ngx, band = (int)blockIdx.x / g.ngx;
+    const int s = gx * BW + warp;
+    if (s >= g.nstrip) return;
+    int y0, y1;
+    band_rows(band, g.nband, g.h, y0, y1);
+    const bool cl = s < g.sx0, cr = s >= g.sx1, cy = band < g.by0 || band >= g.by1;
+    const uint32_t ring = su32(rings[warp]);
+    if (cy) fused_band_body<true>(p, ring, s * FSTRIP, y0, y1 - y0, lane, cl, cr);
+    else fused_band_body<false>(p, ring, s * FSTRIP, y0, y1 - y0, lane, cl, cr);
+}
+
 int num_sms()
 {
     static int n = 0;
@@ -540,12 +804,12 @@ int band_nw()
 
 const void *lap_band_fn(int nw) { return nw == 2 ? (const void *)k_lap_band<2> : (const void *)k_lap_band<4>; }
 
-// resident CTAs per SM: which = 2 / 4 (Laplace, NW words per lane), 1 (Harris)
+// resident CTAs per SM: which = 2 / 4 (Laplace, NW words per lane), 1 (Harris), 3 (fused cfg3)
 int band_blocks_per_sm(int which)
 {
     static int nb[5] = {-1, -1, -1, -1, -1};
     if (nb[which] < 0) {
-        const void *fn = which == 1 ? (const void *)k_har_band : lap_band_fn(which);
+        const void *fn = which == 1 ? (const void *)k_har_band : which == 3 ? (const void *)k_fused_band : lap_band_fn(which);
         if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb[which], fn, NTB, 0) != cudaSuccess) {
             cudaGetLastError();
             nb[which] = 0;
@@ -666,4 +930,32 @@ cudaError_t ispi_harris_band(const int16_t *dx, const int16_t *dy, int w, int h,
     p.thr_err = 2.0f * 5.9604645e-08f * std::fabs(p.thr_f) + 1e-30f;   // |(float)thr - thr| + margin
     bounds[0] = p.g.sx0; bounds[1] = std::max(p.g.sx0, p.g.sx1); bounds[2] = p.g.by0; bounds[3] = p.g.by1;
     return launch_band((const void *)k_har_band, &p, p.g.ngx * p.g.nband, st);
+}
+
+// Fused cfg3 band kernel: 4-pixel lane granules, 4-byte aligned rows in and out (8-byte for
+// the optional dx / dy), h >= 8.
+bool ispi_band_fused_ok(const void *img, int w, int h, int pitch, const void *mag, const void *lap, const void *har,
+                        const void *dx, const void *dy, int out_pitch)
+{
+    auto al = [](const void *q, long long pb, int a) { return ((uintptr_t)q % a) == 0 && (pb % a) == 0; };
+    return al(img, pitch, 4) && al(mag, out_pitch, 4) && al(lap, out_pitch, 4) && al(har, out_pitch, 4) &&
+           (!dx || al(dx, 2LL * out_pitch, 8)) && (!dy || al(dy, 2LL * out_pitch, 8)) && (!dx == !dy) && w % 4 == 0 &&
+           w >= 8 && h >= 8;
+}
+
+cudaError_t ispi_fused_band(const uint8_t *img, int w, int h, int pitch, int mode, int cval, int hcval, long long thr,
+                            int16_t *dx, int16_t *dy, uint8_t *mag, uint8_t *lap, uint8_t *har, int out_pitch,
+                            cudaStream_t st)
+{
+    FusedBandParams p{};
+    p.g = band_geom(w, h, pitch, out_pitch, mode, 2, FSTRIP, band_blocks_per_sm(3), bands_hint());
+    p.img = img;
+    p.mag = mag; p.lap = lap; p.har = har; p.dx = dx; p.dy = dy;
+    p.cword = 0x01010101u * (uint32_t)(cval & 0xff);
+    p.hcf = (float)hcval;
+    p.c4 = 4.0f * (float)hcval * (float)hcval;
+    p.thr = (double)std::max(-9007199254740992ll, std::min(9007199254740992ll, thr));
+    p.thr_f = (float)p.thr;
+    p.thr_err = 2.0f * 5.9604645e-08f * std::fabs(p.thr_f) + 1e-30f;
+    return launch_band((const void *)k_fused_band, &p, p.g.ngx * p.g.nband, st);
 }

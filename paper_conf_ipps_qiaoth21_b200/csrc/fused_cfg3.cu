@@ -758,8 +758,15 @@ extern "C" isp_status_t isp_pipeline_cfg3_u8(const uint8_t *img, int w, int h, i
     // reflections suffice at its borders); ISP_NAIVE, unaligned or tiny images: the general kernel
     const bool body = !p.naive && p.vec && p.vec_out && p.bx1 > p.bx0 && p.by1 > p.by0 && w >= 2 * TW && h >= 2 * TH &&
                       !getenv("ISP_FUSED_V1");
+    // ISP_AUTO / ISP_TMA: the warp-strip band kernel (band_u8.cu) when eligible;
+    // ISP_BLOCK / ISP_WARP: the tile-ISP kernel above; ISP_NAIVE: the general kernel
+    const bool band = (variant == ISP_AUTO || variant == ISP_TMA) &&
+                      ispi_band_fused_ok(img, w, h, pitch, mag, lap, harris, dx, dy, out_pitch);
     cudaError_t e = cudaSuccess;
-    if (body) {
+    if (band) {
+        e = ispi_fused_band(img, w, h, pitch, border_mode, const_val, harris_const, thr, dx, dy, mag, lap, harris,
+                            out_pitch, (cudaStream_t)stream);
+    } else if (body) {
         static bool attr = false;
         if (!attr) {
             cudaFuncSetAttribute(k_fused_body, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(BodySmem));
@@ -769,7 +776,7 @@ extern "C" isp_status_t isp_pipeline_cfg3_u8(const uint8_t *img, int w, int h, i
     } else {
         k_fused_cfg3<<<dim3(nbx, nby), NT, 0, (cudaStream_t)stream>>>(p);
     }
-    e = cudaGetLastError();
+    if (e == cudaSuccess) e = cudaGetLastError();
     if (e != cudaSuccess) return ispi_fail(ISP_ECUDA, "isp_pipeline_cfg3_u8: %s", cudaGetErrorString(e));
     return ISP_OK;
 }

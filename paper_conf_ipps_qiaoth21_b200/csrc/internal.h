@@ -45,3 +45,8 @@ cudaError_t ispi_harris_band(const int16_t *dx, const int16_t *dy, int w, int h,
                              long long thr, uint8_t *out, int out_pitch, cudaStream_t st, int bounds[4]);
 cudaError_t ispi_laplace_band(const uint8_t *img, int w, int h, int pitch, int mode, int cval, uint8_t *out,
                               int out_pitch, cudaStream_t st, int bounds[4]);
+bool ispi_band_fused_ok(const void *img, int w, int h, int pitch, const void *mag, const void *lap, const void *har,
+                        const void *dx, const void *dy, int out_pitch);
+cudaError_t ispi_fused_band(const uint8_t *img, int w, int h, int pitch, int mode, int cval, int hcval, long long thr,
+                            int16_t *dx, int16_t *dy, uint8_t *mag, uint8_t *lap, uint8_t *har, int out_pitch,
+                            cudaStream_t st);

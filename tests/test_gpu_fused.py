@@ -41,15 +41,19 @@ def composition(img, mode, c, hc, thr):
     return rdx, rdy, rmag, oracle.laplace5_u8(img, mode, c), oracle.harris(rdx, rdy, mode, hc, thr)
 
 
-@pytest.mark.parametrize("shape", [(1, 1), (2, 3), (5, 130), (33, 129), (64, 64), (70, 300), (131, 517)])
+@pytest.mark.parametrize("shape", [(1, 1), (2, 3), (5, 130), (33, 129), (64, 64), (70, 300), (131, 517), (8, 8),
+                                   (9, 132), (70, 2064), (45, 260), (300, 1000)])
 @pytest.mark.parametrize("kind", ["structured", "noise"])
 def test_fused_matches_composition(isp, shape, kind):
+    """auto / tma: the band kernel where w % 4 == 0 and h >= 8 (partial strips down to one
+    lane, single-strip images, bands holding both image edges), else the tile / general
+    kernels; warp: the tile-ISP kernel; naive: the general kernel."""
     h, w = shape
     img = synth.structured_u8(h, w, 5) if kind == "structured" else synth.uniform_u8(h, w, 5)
     d = dev(img)
     for mode in MODES:
         rdx, rdy, rmag, rlap, rhar = composition(img, mode, 45, -3, 0)
-        for v in ["auto", "naive"]:
+        for v in ["auto", "tma", "warp", "naive"]:
             dx = torch.empty((h, w), dtype=torch.int16, device="cuda")
             dy = torch.empty_like(dx)
             mag, lap, har = isp.isp_pipeline_cfg3_u8(d, mode, 45, -3, 0, dx=dx, dy=dy, variant=v)
