@@ -456,7 +456,8 @@ def run_isp(args):
             "frac": achieved / (hbm if hbm else 6650.0),
             "peak_source": "MEASURED_PEAKS.json hbm_gbs (measured)" if hbm else "fallback (B200_PROFILING.md)",
             "kernel": f"variant {args.variant}: " + (
-                (f"k_pstaged<{kname}> (persistent TMA-staged ISP)" if os.environ.get("ISP_TMA_PERSIST") == "1"
+                (f"k_sep_band<{wl.window}> (warp-strip band ISP, cp.async ring; band_f32.cu)" if plan["tile_w"] == 128
+                 else f"k_pstaged<{kname}> (persistent TMA-staged ISP)" if os.environ.get("ISP_TMA_PERSIST") == "1"
                  else f"k_staged<{kname}> (TMA-staged ISP)") if plan["choice"] == 4 else f"k_stencil<{kname}>"),
             "algorithmic_bytes_per_launch": rank_bytes,
             "duration_us": per_launch_us,

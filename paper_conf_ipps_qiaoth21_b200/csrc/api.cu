@@ -651,7 +651,8 @@ isp_status_t resolve_and_launch(Desc &d, int fam, int w, int h, int mw, int mh, 
 // = 0) and Harris (1): ISP_TMA runs them when eligible; ISP_AUTO evaluates Eq. (10) for
 // them (form S, reading A21, calibrated constants, occupancy from the API) against the
 // naive kernel.  Returns false when the caller should take the generic path.
-// which = 2 / 3: the Laplace / Harris band kernels (band_u8.cu: warp strips x bands of rows)
+// which = 2 / 3: the Laplace / Harris band kernels (band_u8.cu: warp strips x bands of rows);
+// 4: the separable f32 band kernel (band_f32.cu)
 bool tile_variant(int which, int fam, int mode, int w, int h, int mw, int mh, isp_variant_t v, bool ok,
                   const std::function<cudaError_t(int *)> &launch, isp_status_t &st, const char *what)
 {
@@ -659,6 +660,7 @@ bool tile_variant(int which, int fam, int mode, int w, int h, int mw, int mh, is
     int tw, th;
     if (which == 2) ispi_band_shape(w, h, &tw, &th);
     else if (which == 3) ispi_band_harris_shape(w, h, &tw, &th);
+    else if (which == 4) ispi_sep_band_shape(w, h, mw, &tw, &th);
     else ispi_tile_shape(&tw, &th);
     Plan p = make_plan(w, h, mw / 2, mh / 2, 4, tw, th, which >= 2 ? tw : 128);
     isp_plan_info info{};
@@ -667,7 +669,8 @@ bool tile_variant(int which, int fam, int mode, int w, int h, int mw, int mh, is
         isp_model_params mp;
         defaults(fam, mode, mp);
         mp.form = 2;
-        const int nb = which >= 2 ? ispi_band_blocks_per_sm(which == 3 ? 1 : 0) : ispi_tile_blocks_per_sm(which);
+        const int nb = which == 4 ? ispi_sep_band_blocks_per_sm(mw)
+                       : which >= 2 ? ispi_band_blocks_per_sm(which == 3 ? 1 : 0) : ispi_tile_blocks_per_sm(which);
         info.o_isp = occupancy_of(nb > 0 ? nb : 1, 128);
         info.o_naive = 0.5;   // the naive streaming kernel (64 regs x 128 threads: 8 blocks / SM)
         model(p, w, h, mw, mh, mp, info);
@@ -932,6 +935,16 @@ isp_status_t ispi_filter_f32(const float *img, int w, int h, int pitch, const fl
         if (separable_f32(mask, mw, mh, row, col)) {
             d.rowf = row.data();
             d.colf = col.data();
+            // ISP_TMA / AUTO on whole images: the warp-strip band kernel (band_f32.cu)
+            isp_status_t ts;
+            if (!rr && !getenv("ISP_F32_STAGED") &&
+                tile_variant(4, F_SEP_F32, border_mode, w, h, mw, mh, variant,
+                             ispi_sep_band_ok(img, w, h, pitch, out, out_pitch, mw, mh),
+                             [&](int *b) { return ispi_sep_band(img, w, h, pitch, row.data(), col.data(), mw,
+                                                               border_mode, const_val, out, out_pitch,
+                                                               (cudaStream_t)stream, b); },
+                             ts, "isp_filter(separable band)"))
+                return ts;
             return resolve_and_launch(d, F_SEP_F32, w, h, mw, mh, mw / 2, mh / 2, false, variant, kfn_sep_f32,
                                       run_sep_f32, "isp_filter(separable)", rr,
                                       aligned(img, (long long)pitch * 4, 16), 4, 1);

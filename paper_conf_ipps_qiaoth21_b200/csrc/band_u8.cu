@@ -32,17 +32,16 @@
 #include "../../include/isp.h"
 #include "internal.h"
 #include "harris_core.cuh"
+#include "band_common.cuh"
 
 namespace {
 
-constexpr int BW = 4;                      // warps per CTA (adjacent strips of one band)
-constexpr int NTB = 32 * BW;
 #ifndef BAND_LAP_D
 #define BAND_LAP_D 5
 #endif
 constexpr int LD = BAND_LAP_D;             // rows in flight per warp
-constexpr int LR = 8;                      // ring slots (power of 2): newest + D in flight
 static_assert(LR >= LD + 1, "ring too small");
+
 
 // NW words (4 pixels each) per lane
 template <int NW> struct BandShape {
@@ -52,46 +51,12 @@ template <int NW> struct BandShape {
     static constexpr int MINB = NW == 2 ? 8 : 5; // resident CTAs per SM (register cap)
 };
 
-struct BandGeom {
-    int w, h, pitch, out_pitch, mode;
-    int nstrip, ngx, nband;  // strips, CTA columns, bands
-    int sx0, sx1, by0, by1;  // Body strips [sx0, sx1), Body bands [by0, by1)
-};
-
 struct LapBandParams {
     BandGeom g;
     const uint8_t *img;
     uint8_t *out;
     uint32_t cword;  // the constant in all four bytes
 };
-
-__device__ __forceinline__ uint32_t su32(const void *p) { return (uint32_t)__cvta_generic_to_shared(p); }
-__device__ __forceinline__ void cpa_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
-template <int N>
-__device__ __forceinline__ void cpa_wait()
-{
-    asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory");
-}
-
-__device__ __forceinline__ void band_rows(int b, int nb, int h, int &y0, int &y1)
-{
-    y0 = (int)((long long)b * h / nb);
-    y1 = (int)((long long)(b + 1) * h / nb);
-}
-
-// Row y through the border pattern for an overshoot of at most the window's
-// reach (one reflection: the launch requires h >= 8); -1: Constant, row outside.
-template <bool CHK>
-__device__ __forceinline__ int map_row1(int y, int h, int mode)
-{
-    if (!CHK || (y >= 0 && y < h)) return y;
-    switch (mode) {
-    case ISP_CLAMP: return y < 0 ? 0 : h - 1;
-    case ISP_MIRROR: return y < 0 ? -y - 1 : 2 * h - 1 - y;
-    case ISP_REPEAT: return y < 0 ? y + h : y - h;
-    default: return -1;
-    }
-}
 
 // cp.async of the lane's NW words, predicated on the lane (lanes past the image copy
 // nothing, so the halo words stored in their positions survive)
@@ -107,20 +72,6 @@ __device__ __forceinline__ void cpa_own(uint32_t dst, const void *src, uint32_t 
                      "l"(src), "r"(on)
                      : "memory");
 }
-// 4-byte cp.async issued only by the lanes with `on` set (a predicated LDGSTS: the other
-// lanes take no part, so the instruction costs one lane of shared-memory traffic)
-__device__ __forceinline__ void cpa4p(uint32_t dst, const void *src, uint32_t on)
-{
-    asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %2, 0;\n\t@q cp.async.ca.shared.global [%0], [%1], 4;\n\t}" ::"r"(dst),
-                 "l"(src), "r"(on)
-                 : "memory");
-}
-__device__ __forceinline__ uint32_t lds32(uint32_t a)
-{
-    uint32_t v;
-    asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(a) : "memory");
-    return v;
-}
 template <int NW>
 __device__ __forceinline__ void lds_own(uint32_t a, uint32_t (&w)[NW])
 {
@@ -129,10 +80,6 @@ __device__ __forceinline__ void lds_own(uint32_t a, uint32_t (&w)[NW])
                      : "memory");
     else
         asm volatile("ld.shared.v2.u32 {%0, %1}, [%2];" : "=r"(w[0]), "=r"(w[1]) : "r"(a) : "memory");
-}
-__device__ __forceinline__ void sts32(uint32_t a, uint32_t v)
-{
-    asm volatile("st.shared.u32 [%0], %1;" ::"r"(a), "r"(v) : "memory");
 }
 // 16-bit pair lanes of a word: (b0, b2) and (b1, b3)
 __device__ __forceinline__ uint32_t ev(uint32_t w) { return __byte_perm(w, 0u, 0x4240); }
@@ -781,20 +728,6 @@ __global__ void __launch_bounds__(NTB, 4) k_fused_band(const __grid_constant__ F
     else fused_band_body<false>(p, ring, s * FSTRIP, y0, y1 - y0, lane, cl, cr);
 }
 
-int num_sms()
-{
-    static int n = 0;
-    if (n == 0) {
-        int dev = 0;
-        if (cudaGetDevice(&dev) != cudaSuccess || cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev) !=
-                                                      cudaSuccess) {
-            cudaGetLastError();
-            n = 148;
-        }
-    }
-    return n;
-}
-
 // Words per lane of the Laplace band launch: 4 (16 pixels) unless ISP_BAND_NW=2
 int band_nw()
 {
@@ -816,53 +749,6 @@ int band_blocks_per_sm(int which)
         }
     }
     return nb[which];
-}
-
-// Strips, bands and the Body rectangle (hy rows of reach; a strip's right halo word lies
-// past it, so a strip is Body iff it ends before the image's last column).
-BandGeom band_geom(int w, int h, int pitch, int out_pitch, int mode, int hy, int strip, int per_sm, int bands_hint)
-{
-    BandGeom g{};
-    g.w = w; g.h = h; g.pitch = pitch; g.out_pitch = out_pitch; g.mode = mode;
-    g.nstrip = (w + strip - 1) / strip;
-    g.ngx = (g.nstrip + BW - 1) / BW;
-    int nb = bands_hint;
-    if (nb <= 0) {
-        nb = std::max(1, num_sms() * std::max(1, per_sm) / g.ngx);
-    }
-    g.nband = std::max(1, std::min(nb, h / (2 * hy + 2)));
-    g.sx0 = 1;
-    g.sx1 = (w - 1) / strip;
-    g.by0 = g.nband;
-    g.by1 = g.nband;
-    for (int b = g.nband - 1; b >= 0; --b) {
-        const int y0 = (int)((long long)b * h / g.nband), y1 = (int)((long long)(b + 1) * h / g.nband);
-        if (y0 >= hy) g.by0 = b;
-        if (y1 + hy > h) g.by1 = b;
-    }
-    if (g.by1 < g.by0) g.by1 = g.by0;
-    return g;
-}
-
-cudaError_t launch_band(const void *fn, void *params, int nblocks, cudaStream_t st)
-{
-    cudaLaunchConfig_t cfg{};
-    cfg.gridDim = dim3(nblocks);
-    cfg.blockDim = dim3(NTB);
-    cfg.stream = st;
-    cudaLaunchAttribute at[1];
-    at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
-    at[0].val.programmaticStreamSerializationAllowed = 1;
-    cfg.attrs = at;
-    cfg.numAttrs = 1;
-    void *args[] = {params};
-    return cudaLaunchKernelExC(&cfg, fn, args);
-}
-
-int bands_hint()
-{
-    const char *e = getenv("ISP_BAND_BANDS");
-    return e ? atoi(e) : 0;
 }
 
 }  // namespace

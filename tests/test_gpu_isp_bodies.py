@@ -86,11 +86,15 @@ def binomial_f32(m):
 
 
 # ---------------------------------------------------------------- f32, compiled windows
+@pytest.mark.parametrize("staged", [False, True])
 @pytest.mark.parametrize("mask_kind", ["binomial3", "binomial5", "binomial7", "rand3", "rand5", "rand7"])
 @pytest.mark.parametrize("shape", F32_SHAPES)
-def test_f32_compiled_bodies(isp, shape, mask_kind):
-    """OpSepF32<3/5/7> (rank-1 masks) and OpConvF32<3/5/7> in k_staged, k_stencil
-    Listing 3 / Listing 5 bodies and naive, every border mode."""
+def test_f32_compiled_bodies(isp, shape, mask_kind, staged, monkeypatch):
+    """OpSepF32<3/5/7> (rank-1 masks) and OpConvF32<3/5/7> in the TMA-staged k_staged
+    (staged, or any non-separable mask) or the band kernel k_sep_band (separable masks),
+    k_stencil Listing 3 / Listing 5 bodies and naive, every border mode."""
+    if staged:
+        monkeypatch.setenv("ISP_F32_STAGED", "1")
     h, w = shape
     img = synth.uniform_f32(h, w, 100 + h)
     m = int(mask_kind[-1])
@@ -105,8 +109,11 @@ def test_f32_compiled_bodies(isp, shape, mask_kind):
             np.testing.assert_array_equal(o, outs["naive"], err_msg=f"{v} != naive ({mode} {mask_kind})")
 
 
+@pytest.mark.parametrize("staged", [False, True])
 @pytest.mark.parametrize("m", [3, 5, 7])
-def test_f32_separable_entry_bodies(isp, m):
+def test_f32_separable_entry_bodies(isp, m, staged, monkeypatch):
+    if staged:
+        monkeypatch.setenv("ISP_F32_STAGED", "1")
     h, w = F32_SHAPES[0]
     img = synth.uniform_f32(h, w, 5)
     rng = np.random.default_rng(m)
@@ -574,3 +581,27 @@ def test_harris_band_kernel(isp, shape):
                     assert p["choice"] == CODE["tma"] and p["warp_w"] == 128 and p["tile_h"] < 32, p
                     np.testing.assert_array_equal(got, oracle.harris(dx, dy, mode, c, thr),
                                                   err_msg=f"{mode} c={c} thr={thr}")
+
+
+# ---------------------------------------------------------------- warp-strip band f32 (separable)
+@pytest.mark.parametrize("m", [3, 5, 7])
+@pytest.mark.parametrize("shape", [(8, 8), (9, 132), (70, 2052), (45, 4100), (300, 520), (4096 // 8, 4096)])
+def test_sep_band_kernel(isp, shape, m):
+    """k_sep_band (band_f32.cu), the TMA / AUTO kernel of whole-image separable f32 masks:
+    strips of 128 columns (partial last strips down to one lane, one strip that is L and R),
+    bands holding both image edges, binomial and random rank-1 masks, every mode -- A28
+    against the oracle and bitwise equal to the naive kernel, the plan showing the band
+    kernel (128-column tiles, TMA choice)."""
+    h, w = shape
+    img = synth.uniform_f32(h, w, 300 + m)
+    rng = np.random.default_rng(77 + m)
+    for mask in (binomial_f32(m), np.outer(rng.standard_normal(m), rng.standard_normal(m)).astype(np.float32)):
+        d = dev(img)
+        for mode in MODES:
+            ref, sc = oracle.filter_f64(img, mask, mode, 0.625, with_scale=True)
+            got = host(isp.isp_filter_ex(d, mask, mode, 0.625, variant="tma"))
+            p = isp.isp_last_plan()
+            assert p["choice"] == CODE["tma"] and p["tile_w"] == 128 and p["warp_w"] == 128, p
+            check_f32(got, ref, sc)
+            naive = host(isp.isp_filter_ex(d, mask, mode, 0.625, variant="naive"))
+            np.testing.assert_array_equal(got, naive, err_msg=f"band != naive {mode} m={m}")
