@@ -639,7 +639,7 @@ def main():
     ap.add_argument("--check-launch", action="store_true", help="only check the N-rank launch path")
     ap.add_argument("--halo", default="peer", choices=["peer", "nccl"],
                     help="N > 1: neighbour rows read from peer memory (default) or exchanged with NCCL")
-    ap.add_argument("--steps", type=int, default=6000)
+    ap.add_argument("--steps", type=int, default=200)
     ap.add_argument("--warmup", type=int, default=20)
     ap.add_argument("--impl", default="isp", choices=["isp", "reference"])
     ap.add_argument("--variant", default="auto", choices=["auto", "tma", "warp", "block", "naive"])
