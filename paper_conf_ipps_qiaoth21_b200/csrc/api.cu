@@ -572,7 +572,9 @@ isp_status_t resolve_and_launch(Desc &d, int fam, int w, int h, int mw, int mh, 
         isp_model_params mp;
         defaults(fam, d.mode, mp);
         info.o_naive = nb_naive > 0 ? occupancy_of(nb_naive, threads) : 1.0;
-        info.o_isp = chosen == ISP_TMA ? occupancy_of(nb_tma, tma_threads)
+        // staged / tiled kernels (TMA): latency is hidden by the staging, not by resident
+        // warps, so their occupancy term is the naive kernel's (reading A34)
+        info.o_isp = chosen == ISP_TMA ? info.o_naive
                                        : (nb_stream > 0 ? occupancy_of(nb_stream, threads) : 1.0);
         n_block(p, info.n_block);
         if (chosen == ISP_TMA) mp.form = 2;   // staged kernels: checks per staged element (A21)
@@ -650,10 +652,14 @@ isp_status_t resolve_and_launch(Desc &d, int fam, int w, int h, int mw, int mh, 
 // The tile-staged u8 / i16 kernels (tile_u8.cu) as the ISP_TMA variant of Laplace (which
 // = 0) and Harris (1): ISP_TMA runs them when eligible; ISP_AUTO evaluates Eq. (10) for
 // them (form S, reading A21, calibrated constants, occupancy from the API) against the
-// naive kernel.  Returns false when the caller should take the generic path.
+// naive kernel.  Returns false when the caller should take the generic path; when AUTO's
+// Eq. (10) rejects the ISP kernel, v becomes ISP_NAIVE (the decision is ISP vs naive, not a
+// cascade through other ISP implementations).
 // which = 2 / 3: the Laplace / Harris band kernels (band_u8.cu: warp strips x bands of rows);
-// 4: the separable f32 band kernel (band_f32.cu)
-bool tile_variant(int which, int fam, int mode, int w, int h, int mw, int mh, isp_variant_t v, bool ok,
+// 4: the separable f32 band kernel (band_f32.cu); 5: the Sobel band kernel.  The band kernels keep several rows in
+// flight per warp, so resident warps do not measure their latency hiding: their occupancy
+// term is taken equal to the naive kernel's (reading A34).
+bool tile_variant(int which, int fam, int mode, int w, int h, int mw, int mh, isp_variant_t &v, bool ok,
                   const std::function<cudaError_t(int *)> &launch, isp_status_t &st, const char *what)
 {
     if (!(v == ISP_TMA || v == ISP_AUTO) || !ok) return false;
@@ -661,6 +667,7 @@ bool tile_variant(int which, int fam, int mode, int w, int h, int mw, int mh, is
     if (which == 2) ispi_band_shape(w, h, &tw, &th);
     else if (which == 3) ispi_band_harris_shape(w, h, &tw, &th);
     else if (which == 4) ispi_sep_band_shape(w, h, mw, &tw, &th);
+    else if (which == 5) ispi_band_sobel_shape(w, h, &tw, &th);
     else ispi_tile_shape(&tw, &th);
     Plan p = make_plan(w, h, mw / 2, mh / 2, 4, tw, th, which >= 2 ? tw : 128);
     isp_plan_info info{};
@@ -669,12 +676,17 @@ bool tile_variant(int which, int fam, int mode, int w, int h, int mw, int mh, is
         isp_model_params mp;
         defaults(fam, mode, mp);
         mp.form = 2;
-        const int nb = which == 4 ? ispi_sep_band_blocks_per_sm(mw)
-                       : which >= 2 ? ispi_band_blocks_per_sm(which == 3 ? 1 : 0) : ispi_tile_blocks_per_sm(which);
-        info.o_isp = occupancy_of(nb > 0 ? nb : 1, 128);
+        const int nb = which == 4   ? ispi_sep_band_blocks_per_sm(mw)
+                       : which == 5 ? ispi_band_blocks_per_sm(2)
+                       : which >= 2 ? ispi_band_blocks_per_sm(which == 3 ? 1 : 0)
+                                    : ispi_tile_blocks_per_sm(which);
         info.o_naive = 0.5;   // the naive streaming kernel (64 regs x 128 threads: 8 blocks / SM)
+        info.o_isp = which >= 2 ? info.o_naive : occupancy_of(nb > 0 ? nb : 1, 128);
         model(p, w, h, mw, mh, mp, info);
-        if (!(info.g > 1.0)) return false;
+        if (!(info.g > 1.0)) {
+            v = ISP_NAIVE;
+            return false;
+        }
     }
     int b[4];
     cudaError_t e = launch(b);
@@ -1107,6 +1119,14 @@ isp_status_t isp_sobel_u8(const uint8_t *img, int w, int h, int pitch, int borde
     d.g.vec_in = aligned(img, pitch, 8);
     d.g.vec_out = (!dx || aligned(dx, 2LL * out_pitch, 16)) && (!dy || aligned(dy, 2LL * out_pitch, 16)) &&
                   (!mag || aligned(mag, out_pitch, 8));
+    // ISP_TMA / AUTO: the band kernel (band_u8.cu) when eligible
+    isp_status_t ts;
+    if (tile_variant(5, F_SOBEL, border_mode, w, h, 3, 3, variant,
+                     ispi_band_sobel_ok(img, w, h, pitch, dx, dy, mag, out_pitch),
+                     [&](int *b) { return ispi_sobel_band(img, w, h, pitch, border_mode, const_val, dx, dy, mag, out_pitch,
+                                                          (cudaStream_t)stream, b); },
+                     ts, "isp_sobel_u8(band)"))
+        return ts;
     return resolve_and_launch(d, F_SOBEL, w, h, 3, 3, 1, 1, false, variant, kfn_sobel, run_sobel, "isp_sobel_u8",
                               nullptr, aligned(img, pitch, 16), 1, 1);
 }

@@ -728,6 +728,148 @@ __global__ void __launch_bounds__(NTB, 4) k_fused_band(const __grid_constant__ F
     else fused_band_body<false>(p, ring, s * FSTRIP, y0, y1 - y0, lane, cl, cr);
 }
 
+
+// ------------------------------------------------------------------------------ Sobel
+// Sobel dx, dy and magnitude (a9) on the same skeleton: 4 pixels per lane, rows y0-1 ..
+// y0+rows streamed once; per row the horizontal parts s = a + 2b + c, d = c - a of the
+// pairs E = (p0, p2), O = (p1, p3) on biased 16-bit lanes, two rows later dx = d + 2d + d,
+// dy = s - s (bias 1024 per lane) -> exact floats -> magnitude (sqrt.approx, §7c) and the
+// int16 images (low halves of v + 1.5 * 2^23).  Any subset of dx / dy / mag is written.
+// Border handling is the staging's (rows mapped at copy time, edge lanes' halo bytes by
+// selectors).  Bit-exact against the oracle.
+struct SobBandParams {
+    BandGeom g;
+    const uint8_t *img;
+    int16_t *dx, *dy;
+    uint8_t *mag;
+    uint32_t cword;
+};
+
+struct SobP { uint32_t sE, sO, dE, dO; };
+
+template <bool CY>
+__device__ __forceinline__ void sob_band_body(const SobBandParams &p, uint32_t ring, int xs0, int y0, int rows,
+                                              int lane, bool cl, bool cr)
+{
+    const BandGeom &g = p.g;
+    constexpr int LPX = 4;
+    const int x = xs0 + LPX * lane;
+    const bool active = !cr || x < g.w;
+    const bool redge = cr && x + LPX == g.w;
+    const int nin = rows + 2;   // >= 6
+    const uint32_t loff = LPX * lane;
+    int acol = xs0 - 4, bcol = xs0 + FSTRIP;
+    uint32_t aon = lane == 0 && (!cl || g.mode == ISP_REPEAT), bdst = 16 + FSTRIP, bon = !cr && lane == 31;
+    if (cl) acol = g.w - 4;
+    if (redge && g.mode == ISP_REPEAT) { bon = 1; bcol = 0; bdst = 16 + LPX * (lane + 1); }
+    uint32_t sl_ = 0x3210, sr_ = 0x3210;
+    if (cl && lane == 0) sl_ = g.mode == ISP_CLAMP ? 0x4444 : g.mode == ISP_MIRROR ? 0x4500 : 0x3210;
+    if (redge) sr_ = g.mode == ISP_CLAMP ? 0x7777 : g.mode == ISP_MIRROR ? 0x0067 : 0x3210;
+    if (g.mode == ISP_CONSTANT) {
+        for (int j = 0; j < LR; ++j) {
+            if (cl && lane == 0) sts32(ring + j * FSLOT + 12, p.cword);
+            if (redge) sts32(ring + j * FSLOT + 16 + LPX * (lane + 1), p.cword);
+        }
+    }
+    const int mcol = active ? x : 0;
+    const uint8_t *nrp = p.img + (ptrdiff_t)(y0 - 1) * g.pitch;
+    auto issue = [&](int j, uint32_t slot) {
+        const uint8_t *rp = nrp;
+        if constexpr (CY) {
+            const int yy = map_row1<true>(y0 - 1 + j, g.h, g.mode);
+            if (yy < 0) {
+                sts32(slot + 16 + loff, p.cword);
+                if (lane == 0) sts32(slot + 12, p.cword);
+                if (lane == 31) sts32(slot + 16 + FSTRIP, p.cword);
+                return;
+            }
+            rp = p.img + (size_t)yy * g.pitch;
+        }
+        cpa4p(slot + 16 + loff, rp + mcol, active);
+        cpa4p(slot + 12, rp + acol, aon);
+        cpa4p(slot + bdst, rp + bcol, bon);
+    };
+#pragma unroll
+    for (int j = 0; j < FLD; ++j) {
+        issue(j, ring + j * FSLOT);
+        nrp += g.pitch;
+        cpa_commit();
+    }
+    SobP sr[3];
+    ptrdiff_t o2 = (ptrdiff_t)(y0 - 2) * g.out_pitch + x;   // output offset of row y0 + i - 2
+#pragma unroll 1
+    for (int i0 = 0; i0 < nin; i0 += 3) {
+#pragma unroll
+        for (int k = 0; k < 3; ++k) {
+            const int i = i0 + k;
+            if (i < nin) {
+                cpa_wait<FLD - 1>();
+                __syncwarp();
+                const uint32_t sl = ring + (i & (LR - 1)) * FSLOT + loff;
+                const uint32_t W0 = lds32(sl + 16);
+                const uint32_t L = __byte_perm(lds32(sl + 12), W0, sl_), R = __byte_perm(lds32(sl + 20), W0, sr_);
+                const uint32_t F0 = __funnelshift_r(L, W0, 16), F1 = __funnelshift_r(W0, R, 16);
+                const uint32_t Om2 = od(F0), E0 = ev(W0), O0 = od(W0), E2 = ev(F1);
+                SobP &sh = sr[k];
+                sh.sE = Om2 + 2u * E0 + O0;
+                sh.sO = E0 + 2u * O0 + E2;
+                sh.dE = O0 + 0x01000100u - Om2;
+                sh.dO = E2 + 0x01000100u - E0;
+                if (i >= 2) {   // row y0 + i - 2 from rows i-2, i-1, i
+                    const SobP &a = sr[(k + 1) % 3], &b = sr[(k + 2) % 3];
+                    const uint32_t dxE = a.dE + 2u * b.dE + sh.dE, dxO = a.dO + 2u * b.dO + sh.dO;
+                    const uint32_t dyE = sh.sE + 0x04000400u - a.sE, dyO = sh.sO + 0x04000400u - a.sO;
+                    const float2 xE = lanes_f(dxE, 1024.f), xO = lanes_f(dxO, 1024.f);
+                    const float2 yE = lanes_f(dyE, 1024.f), yO = lanes_f(dyO, 1024.f);
+                    if (p.mag) {
+                        const float2 nE = fma2(xE, xE, mul2(yE, yE)), nO = fma2(xO, xO, mul2(yO, yO));
+                        const uint32_t m0 = mag_bits(nE.x), m1 = mag_bits(nO.x), m2 = mag_bits(nE.y), m3 = mag_bits(nO.y);
+                        const uint32_t mw =
+                            __byte_perm(__byte_perm(m0, m1, 0x0040), __byte_perm(m2, m3, 0x0040), 0x5410);
+                        if (active) *reinterpret_cast<uint32_t *>(p.mag + o2) = mw;
+                    }
+                    if (p.dx) {   // int16 = low half of the bits of v + 1.5 * 2^23
+                        const float2 a2 = add2(xE, f2(12582912.f, 12582912.f)), b2 = add2(xO, f2(12582912.f, 12582912.f));
+                        if (active)
+                            *reinterpret_cast<uint2 *>(p.dx + o2) =
+                                make_uint2(__byte_perm(__float_as_uint(a2.x), __float_as_uint(b2.x), 0x5410),
+                                           __byte_perm(__float_as_uint(a2.y), __float_as_uint(b2.y), 0x5410));
+                    }
+                    if (p.dy) {
+                        const float2 a2 = add2(yE, f2(12582912.f, 12582912.f)), b2 = add2(yO, f2(12582912.f, 12582912.f));
+                        if (active)
+                            *reinterpret_cast<uint2 *>(p.dy + o2) =
+                                make_uint2(__byte_perm(__float_as_uint(a2.x), __float_as_uint(b2.x), 0x5410),
+                                           __byte_perm(__float_as_uint(a2.y), __float_as_uint(b2.y), 0x5410));
+                    }
+                }
+                o2 += g.out_pitch;
+                if (i + FLD < nin) issue(i + FLD, ring + ((i + FLD) & (LR - 1)) * FSLOT);
+                nrp += g.pitch;
+                cpa_commit();
+            }
+        }
+    }
+}
+
+__global__ void __launch_bounds__(NTB, 8) k_sob_band(const __grid_constant__ SobBandParams p)
+{
+    __shared__ __align__(16) uint8_t rings[BW][LR * FSLOT];
+    asm volatile("griddepcontrol.wait;" ::: "memory");
+    asm volatile("griddepcontrol.launch_dependents;");
+    const BandGeom &g = p.g;
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int gx = (int)blockIdx.x % g.ngx, band = (int)blockIdx.x / g.ngx;
+    const int s = gx * BW + warp;
+    if (s >= g.nstrip) return;
+    int y0, y1;
+    band_rows(band, g.nband, g.h, y0, y1);
+    const bool cl = s < g.sx0, cr = s >= g.sx1, cy = band < g.by0 || band >= g.by1;
+    const uint32_t ring = su32(rings[warp]);
+    if (cy) sob_band_body<true>(p, ring, s * FSTRIP, y0, y1 - y0, lane, cl, cr);
+    else sob_band_body<false>(p, ring, s * FSTRIP, y0, y1 - y0, lane, cl, cr);
+}
+
 // Words per lane of the Laplace band launch: 4 (16 pixels) unless ISP_BAND_NW=2
 int band_nw()
 {
@@ -737,12 +879,16 @@ int band_nw()
 
 const void *lap_band_fn(int nw) { return nw == 2 ? (const void *)k_lap_band<2> : (const void *)k_lap_band<4>; }
 
-// resident CTAs per SM: which = 2 / 4 (Laplace, NW words per lane), 1 (Harris), 3 (fused cfg3)
+// resident CTAs per SM: which = 2 / 4 (Laplace, NW words per lane), 1 (Harris), 3 (fused cfg3),
+// 0 (Sobel)
 int band_blocks_per_sm(int which)
 {
     static int nb[5] = {-1, -1, -1, -1, -1};
     if (nb[which] < 0) {
-        const void *fn = which == 1 ? (const void *)k_har_band : which == 3 ? (const void *)k_fused_band : lap_band_fn(which);
+        const void *fn = which == 1   ? (const void *)k_har_band
+                         : which == 3 ? (const void *)k_fused_band
+                         : which == 0 ? (const void *)k_sob_band
+                                      : lap_band_fn(which);
         if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb[which], fn, NTB, 0) != cudaSuccess) {
             cudaGetLastError();
             nb[which] = 0;
@@ -772,7 +918,7 @@ void ispi_band_shape(int w, int h, int *tw, int *th)
     *th = (h + g.nband - 1) / g.nband;
 }
 
-int ispi_band_blocks_per_sm(int which) { return band_blocks_per_sm(which == 1 ? 1 : band_nw()); }
+int ispi_band_blocks_per_sm(int which) { return band_blocks_per_sm(which == 1 ? 1 : which == 2 ? 0 : band_nw()); }
 
 cudaError_t ispi_laplace_band(const uint8_t *img, int w, int h, int pitch, int mode, int cval, uint8_t *out,
                               int out_pitch, cudaStream_t st, int bounds[4])
@@ -844,4 +990,33 @@ cudaError_t ispi_fused_band(const uint8_t *img, int w, int h, int pitch, int mod
     p.thr_f = (float)p.thr;
     p.thr_err = 2.0f * 5.9604645e-08f * std::fabs(p.thr_f) + 1e-30f;
     return launch_band((const void *)k_fused_band, &p, p.g.ngx * p.g.nband, st);
+}
+
+// Sobel band kernel: 4-pixel lane granules, 4-byte aligned input rows, 4-byte aligned mag
+// rows and 8-byte aligned dx / dy rows, h >= 8.
+bool ispi_band_sobel_ok(const void *img, int w, int h, int pitch, const void *dx, const void *dy, const void *mag,
+                        int out_pitch)
+{
+    auto al = [](const void *q, long long pb, int a) { return ((uintptr_t)q % a) == 0 && (pb % a) == 0; };
+    return al(img, pitch, 4) && (!mag || al(mag, out_pitch, 4)) && (!dx || al(dx, 2LL * out_pitch, 8)) &&
+           (!dy || al(dy, 2LL * out_pitch, 8)) && w % 4 == 0 && w >= 8 && h >= 8;
+}
+
+void ispi_band_sobel_shape(int w, int h, int *tw, int *th)
+{
+    const BandGeom g = band_geom(w, h, w, w, ISP_CLAMP, 1, FSTRIP, band_blocks_per_sm(0), bands_hint());
+    *tw = FSTRIP;
+    *th = (h + g.nband - 1) / g.nband;
+}
+
+cudaError_t ispi_sobel_band(const uint8_t *img, int w, int h, int pitch, int mode, int cval, int16_t *dx, int16_t *dy,
+                            uint8_t *mag, int out_pitch, cudaStream_t st, int bounds[4])
+{
+    SobBandParams p{};
+    p.g = band_geom(w, h, pitch, out_pitch, mode, 1, FSTRIP, band_blocks_per_sm(0), bands_hint());
+    p.img = img;
+    p.dx = dx; p.dy = dy; p.mag = mag;
+    p.cword = 0x01010101u * (uint32_t)(cval & 0xff);
+    bounds[0] = p.g.sx0; bounds[1] = std::max(p.g.sx0, p.g.sx1); bounds[2] = p.g.by0; bounds[3] = p.g.by1;
+    return launch_band((const void *)k_sob_band, &p, p.g.ngx * p.g.nband, st);
 }

@@ -38,7 +38,7 @@ cudaError_t ispi_harris_tile(const int16_t *dx, const int16_t *dy, int w, int h,
 // warp-strip streaming band kernels (band_u8.cu): the ISP_TMA variant of Laplace and Harris
 bool ispi_band_ok(const void *in, int w, int h, int pitch, const void *out, int out_pitch);
 void ispi_band_shape(int w, int h, int *tw, int *th);
-int ispi_band_blocks_per_sm(int which);   // 0: Laplace, 1: Harris
+int ispi_band_blocks_per_sm(int which);   // 0: Laplace, 1: Harris, 2: Sobel
 bool ispi_band_harris_ok(const void *dx, const void *dy, int w, int h, int pitch, const void *out, int out_pitch);
 void ispi_band_harris_shape(int w, int h, int *tw, int *th);
 cudaError_t ispi_harris_band(const int16_t *dx, const int16_t *dy, int w, int h, int pitch, int mode, int cval,
@@ -56,3 +56,8 @@ bool ispi_sep_band_ok(const float *img, int w, int h, int pitch, const float *ou
 void ispi_sep_band_shape(int w, int h, int k, int *tw, int *th);
 cudaError_t ispi_sep_band(const float *img, int w, int h, int pitch, const float *row, const float *col, int k,
                           int mode, float cval, float *out, int out_pitch, cudaStream_t st, int bounds[4]);
+bool ispi_band_sobel_ok(const void *img, int w, int h, int pitch, const void *dx, const void *dy, const void *mag,
+                        int out_pitch);
+void ispi_band_sobel_shape(int w, int h, int *tw, int *th);
+cudaError_t ispi_sobel_band(const uint8_t *img, int w, int h, int pitch, int mode, int cval, int16_t *dx, int16_t *dy,
+                            uint8_t *mag, int out_pitch, cudaStream_t st, int bounds[4]);

@@ -605,3 +605,27 @@ def test_sep_band_kernel(isp, shape, m):
             check_f32(got, ref, sc)
             naive = host(isp.isp_filter_ex(d, mask, mode, 0.625, variant="naive"))
             np.testing.assert_array_equal(got, naive, err_msg=f"band != naive {mode} m={m}")
+
+
+# ---------------------------------------------------------------- warp-strip band Sobel
+@pytest.mark.parametrize("shape", [(8, 8), (9, 132), (70, 2064), (45, 260), (4096 // 8, 4096)])
+def test_sobel_band_kernel(isp, shape):
+    """k_sob_band (band_u8.cu), the TMA / AUTO kernel of isp_sobel_u8: strips of 128
+    columns (partial last strips down to one lane, one strip that is L and R), all modes and
+    constants 0 / 255, every subset of the dx / dy / mag outputs -- bit-exact against the
+    oracle, the plan showing the band kernel."""
+    h, w = shape
+    img = synth.structured_u8(h, w, 41)
+    img[0, :] = 255
+    img[:, -1] = 3
+    d = dev(img)
+    for mode in MODES:
+        for c in ((0, 255) if mode == "constant" else (17,)):
+            rdx, rdy, rmag = oracle.sobel(img, mode, c)
+            for want in (("dx", "dy", "mag"), ("mag",), ("dx",), ("dy", "mag")):
+                dx, dy, mag = isp.isp_sobel_u8(d, mode, c, variant="tma", want=want)
+                p = isp.isp_last_plan()
+                assert p["choice"] == CODE["tma"] and p["warp_w"] == 128 and p["tile_h"] < 32, p
+                for name, got, ref in (("dx", dx, rdx), ("dy", dy, rdy), ("mag", mag, rmag)):
+                    if name in want:
+                        np.testing.assert_array_equal(host(got), ref, err_msg=f"{name} {mode} c={c} {want}")
