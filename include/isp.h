@@ -182,7 +182,8 @@ typedef struct {
 /* Model inputs.  n_check / n_kernel: instructions per border check / per tap of the
  * kernel; ipc_switch: instructions per Listing-3 compare (A18); o_*: occupancy
  * in [0,1] -- pass <= 0 to query the CUDA occupancy API for the kernels this library
- * would launch (needs a GPU).  form: 0 = per-thread switch (A14 "T"), 1 = as printed. */
+ * would launch (needs a GPU).  form: 0 = per-thread switch (A14 "T"), 1 = as printed,
+ * 2 = staged (checks per staged element, A21), 3 = band (checks per staged row, A34). */
 typedef struct {
     double n_check, n_kernel, ipc_switch, o_naive, o_isp;
     int form;

@@ -260,7 +260,12 @@ void model(const Plan &p, int w, int h, int mw, int mh, const isp_model_params &
             const double nb = cols[cc] * brows[rc];
             const double pix = cols[cc] * tx * rows[rc];
             if (mp.form == 1) nisp += (nsw + nreg) * m * n * pix;
-            else if (mp.form == 2) {
+            else if (mp.form == 3) {
+                // band kernels (reading A34): a checked side costs one check per staged row per
+                // thread of the warp (T / B: the row map; L / R: the edge lanes' halo word)
+                const double srows = nb > 0 ? rows[rc] + 2.0 * hy * brows[rc] : 0.0;
+                nisp += nsw * threads * nb + nchk * c * threads * srows * cols[cc] + k * m * n * pix;
+            } else if (mp.form == 2) {
                 const double E = cols[cc] * (tx + 2.0 * hx) * (rows[rc] + 2.0 * hy * brows[rc]);
                 nisp += nsw * threads * nb + nchk * c * E + k * m * n * pix;
             } else nisp += nsw * threads * nb + nreg * m * n * pix;
@@ -675,7 +680,7 @@ bool tile_variant(int which, int fam, int mode, int w, int h, int mw, int mh, is
     if (v == ISP_AUTO) {
         isp_model_params mp;
         defaults(fam, mode, mp);
-        mp.form = 2;
+        mp.form = which >= 2 ? 3 : 2;   // band form (A34) / staged form S (A21)
         const int nb = which == 4   ? ispi_sep_band_blocks_per_sm(mw)
                        : which == 5 ? ispi_band_blocks_per_sm(2)
                        : which >= 2 ? ispi_band_blocks_per_sm(which == 3 ? 1 : 0)

@@ -159,7 +159,7 @@ def _balanced_y0s(h, ny, edge_w=64):
 
 
 @pytest.mark.parametrize("w,h,m", [(4096, 4096, 5), (2048, 1000, 7), (1000, 4096, 13), (4096, 512, 3)])
-@pytest.mark.parametrize("form", [0, 1, 2])
+@pytest.mark.parametrize("form", [0, 1, 2, 3])
 def test_model_balanced_split_matches_oracle(w, h, m, form):
     """Balanced one-wave plans (tile_h = 0): bounds from the real block-row starts and the
     model counting each block's real rows (round-1 counted 0 pixels per block there)."""
@@ -169,17 +169,20 @@ def test_model_balanced_split_matches_oracle(w, h, m, form):
     b = P.bounds_rows(w, h, m, m, 512, y0s)
     assert (got["bh_t"], got["bh_b"], got["nx"], got["ny"]) == (b["BH_T"], b["BH_B"], b["NX"], b["NY"])
     ref = P.model(w, h, m, m, 512, None, 4.0, 20.0, o_naive=0.75, o_isp=0.5, ipc_switch=2.0,
-                  form="TPS"[form], threads_per_block=32, y0s=y0s)
+                  form="TPSB"[form], threads_per_block=32, y0s=y0s)
     for k_got, k_ref in [("n_naive", "N_naive"), ("n_isp", "N_ISP"), ("r_reduced", "R_reduced"), ("g", "G")]:
         assert got[k_got] == pytest.approx(ref[k_ref], rel=1e-12), k_got
     assert got["n_isp"] > 0 and got["g"] < 100      # round 1: pix = 0 made G ~ 855
 
 
-def test_model_form_s_matches_oracle():
-    mp = isp.ModelParams(4.0, 20.0, 2.0, 0.75, 0.5, 2)
-    for (w, m, tw, th) in [(512, 13, 32, 4), (2048, 13, 128, 1), (4096, 5, 512, 32), (4096, 7, 1024, 16)]:
+@pytest.mark.parametrize("form", [2, 3])
+def test_model_form_s_matches_oracle(form):
+    """Forms S (staged, A21) and B (band, A34) of the C model against the oracle planner."""
+    mp = isp.ModelParams(4.0, 20.0, 2.0, 0.75, 0.5, form)
+    for (w, m, tw, th) in [(512, 13, 32, 4), (2048, 13, 128, 1), (4096, 5, 512, 32), (4096, 7, 1024, 16),
+                           (4096, 5, 128, 19), (1000, 3, 128, 7)]:
         got = isp.isp_plan(w, w, m, m, tile_w=tw, tile_h=th, warp_w=tw, params=mp)
-        ref = P.model(w, w, m, m, tw, th, 4.0, 20.0, o_naive=0.75, o_isp=0.5, ipc_switch=2.0, form="S",
+        ref = P.model(w, w, m, m, tw, th, 4.0, 20.0, o_naive=0.75, o_isp=0.5, ipc_switch=2.0, form="SB"[form - 2],
                       threads_per_block=32)
         assert got["n_isp"] == pytest.approx(ref["N_ISP"], rel=1e-12)
         assert got["g"] == pytest.approx(ref["G"], rel=1e-12)

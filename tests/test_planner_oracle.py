@@ -271,6 +271,29 @@ def test_model_form_s_closed_form():
     assert a["N_ISP"] == pytest.approx(b["N_ISP"], rel=1e-12)
 
 
+def test_model_form_b_closed_form():
+    """Form B (reading A34, band kernels) on a 3x3-block image: the 8 border blocks pay
+    n_check per STAGED ROW (ty + 2hy) per thread for each checked side (corners 2, edges 1),
+    Body none -- written out by hand; and an 8x8 image of 2x2 corner blocks counted term by
+    term (A18 switch costs TL 2, TR 3, BL 6, BR 8)."""
+    sx = sy = 48
+    m = n = 5
+    tx = ty = 16
+    c, k, ipc, thr = 3.0, 7.0, 2.0, 64
+    got = P.model(sx, sy, m, n, tx, ty, c, k, ipc_switch=ipc, form="B", threads_per_block=thr)
+    sw = P.n_switch_table()
+    want = sum(sw[r] * ipc * thr for r in P.REGIONS) + (4 * 2 + 4 * 1) * c * thr * (ty + 4) + \
+        9 * k * m * n * tx * ty
+    assert got["N_ISP"] == pytest.approx(want, rel=1e-12)
+    small = P.model(8, 8, 3, 3, 4, 4, 1.0, 1.0, ipc_switch=2.0, form="B")   # threads = tx * ty = 16
+    assert small["N_ISP"] == pytest.approx((2 + 3 + 6 + 8) * 2 * 16 + 4 * 2 * 1 * 16 * 6 + 4 * 9 * 16, rel=1e-12)
+    assert small["N_naive"] == 5 * 9 * 64
+    # with n_check = 0 form B equals form T with n_check = 0 (only the checks differ)
+    a = P.model(sx, sy, m, n, tx, ty, 0.0, k, form="B", threads_per_block=thr)
+    b = P.model(sx, sy, m, n, tx, ty, 0.0, k, form="T", threads_per_block=thr)
+    assert a["N_ISP"] == pytest.approx(b["N_ISP"], rel=1e-12)
+
+
 # ---------------------------------------------------------------- N3: sparse masks (reading A31)
 def test_mask_reach_examples():
     m = np.zeros((7, 7))
