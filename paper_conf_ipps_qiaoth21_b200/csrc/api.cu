@@ -661,7 +661,7 @@ isp_status_t resolve_and_launch(Desc &d, int fam, int w, int h, int mw, int mh, 
 // Eq. (10) rejects the ISP kernel, v becomes ISP_NAIVE (the decision is ISP vs naive, not a
 // cascade through other ISP implementations).
 // which = 2 / 3: the Laplace / Harris band kernels (band_u8.cu: warp strips x bands of rows);
-// 4: the separable f32 band kernel (band_f32.cu); 5: the Sobel band kernel.  The band kernels keep several rows in
+// 4: the separable f32 band kernel (band_f32.cu); 5: Sobel; 6: separable u8.  The band kernels keep several rows in
 // flight per warp, so resident warps do not measure their latency hiding: their occupancy
 // term is taken equal to the naive kernel's (reading A34).
 bool tile_variant(int which, int fam, int mode, int w, int h, int mw, int mh, isp_variant_t &v, bool ok,
@@ -673,6 +673,7 @@ bool tile_variant(int which, int fam, int mode, int w, int h, int mw, int mh, is
     else if (which == 3) ispi_band_harris_shape(w, h, &tw, &th);
     else if (which == 4) ispi_sep_band_shape(w, h, mw, &tw, &th);
     else if (which == 5) ispi_band_sobel_shape(w, h, &tw, &th);
+    else if (which == 6) ispi_sepu8_band_shape(w, h, mw, &tw, &th);
     else ispi_tile_shape(&tw, &th);
     Plan p = make_plan(w, h, mw / 2, mh / 2, 4, tw, th, which >= 2 ? tw : 128);
     isp_plan_info info{};
@@ -683,11 +684,21 @@ bool tile_variant(int which, int fam, int mode, int w, int h, int mw, int mh, is
         mp.form = which >= 2 ? 3 : 2;   // band form (A34) / staged form S (A21)
         const int nb = which == 4   ? ispi_sep_band_blocks_per_sm(mw)
                        : which == 5 ? ispi_band_blocks_per_sm(2)
+                       : which == 6 ? ispi_sepu8_band_blocks_per_sm(mw)
                        : which >= 2 ? ispi_band_blocks_per_sm(which == 3 ? 1 : 0)
                                     : ispi_tile_blocks_per_sm(which);
         info.o_naive = 0.5;   // the naive streaming kernel (64 regs x 128 threads: 8 blocks / SM)
         info.o_isp = which >= 2 ? info.o_naive : occupancy_of(nb > 0 ? nb : 1, 128);
         model(p, w, h, mw, mh, mp, info);
+        if (which >= 2 && p.degenerate) {
+            // a band kernel runs one-strip / one-band images too (its edge warps check both
+            // sides): form B with every side of every block checked
+            const double c = mp.n_check, k = mp.n_kernel, thr = 32.0 * p.wx;
+            const double nb = (double)p.nx * p.ny, srows = (double)h + 2.0 * (mh / 2) * p.ny;
+            info.n_isp = 8.0 * mp.ipc_switch * thr * nb + 4.0 * c * thr * srows * p.nx + k * mw * mh * (double)w * h;
+            info.r_reduced = info.n_naive / info.n_isp;
+            info.g = info.r_reduced * info.o_isp / info.o_naive;
+        }
         if (!(info.g > 1.0)) {
             v = ISP_NAIVE;
             return false;
@@ -956,7 +967,8 @@ isp_status_t ispi_filter_f32(const float *img, int w, int h, int pitch, const fl
             isp_status_t ts;
             if (!rr && !getenv("ISP_F32_STAGED") &&
                 tile_variant(4, F_SEP_F32, border_mode, w, h, mw, mh, variant,
-                             ispi_sep_band_ok(img, w, h, pitch, out, out_pitch, mw, mh),
+                             ispi_sep_band_ok(img, w, h, pitch, out, out_pitch, mw, mh) &&
+                                 (variant == ISP_TMA || ispi_sep_band_fills(w, h, mw)),
                              [&](int *b) { return ispi_sep_band(img, w, h, pitch, row.data(), col.data(), mw,
                                                                border_mode, const_val, out, out_pitch,
                                                                (cudaStream_t)stream, b); },
@@ -1023,6 +1035,17 @@ isp_status_t ispi_filter_u8(const uint8_t *img, int w, int h, int pitch, const i
         if (separable_i32(mask, mw, mh, row, col)) {
             d.rowi = row.data();
             d.coli = col.data();
+            // ISP_TMA / AUTO on whole images: the band kernel (band_u8.cu) for normalised
+            // non-negative masks with a power-of-two divisor (the binomial Gaussians)
+            isp_status_t ts;
+            if (!rr && tile_variant(6, F_U8, border_mode, w, h, mw, mh, variant,
+                                    ispi_sepu8_band_ok(img, w, h, pitch, out, out_pitch, mw, row.data(), col.data(),
+                                                       divisor),
+                                    [&](int *b) { return ispi_sepu8_band(img, w, h, pitch, mw, row.data(), col.data(),
+                                                                         divisor, border_mode, const_val, out,
+                                                                         out_pitch, (cudaStream_t)stream, b); },
+                                    ts, "isp_filter_u8(separable band)"))
+                return ts;
             return resolve_and_launch(d, F_U8, w, h, mw, mh, mw / 2, mh / 2, false, variant, kfn_sep_u8,
                                       run_sep_u8, "isp_filter_u8(separable)", rr, aligned(img, pitch, 16), 1, 1);
         }

@@ -254,15 +254,18 @@ int ispi_sep_band_blocks_per_sm(int k) { return sep_band_blocks_per_sm(k); }
 
 // Eligibility: square separable 3 / 5 / 7 masks, 16-byte aligned rows in and out, w % 4 == 0,
 // h >= 8 (one reflection at every edge), the whole image (no strips).
-// The launch must also give every SM a CTA (ngx x bands >= SMs): narrower images run the
-// TMA-staged / streaming kernels (measured faster at 512^2).
 bool ispi_sep_band_ok(const float *img, int w, int h, int pitch, const float *out, int out_pitch, int mw, int mh)
 {
     auto al = [](const void *q, long long pb) { return ((uintptr_t)q % 16) == 0 && (pb % 16) == 0; };
-    if (!(mw == mh && (mw == 3 || mw == 5 || mw == 7) && al(img, 4LL * pitch) && al(out, 4LL * out_pitch) &&
-          w % 4 == 0 && w >= 8 && h >= 8))
-        return false;
-    const BandGeom g = band_geom(w, h, w, w, ISP_CLAMP, mw / 2, SSTRIP, sep_band_blocks_per_sm(mw), bands_hint(), 185);
+    return mw == mh && (mw == 3 || mw == 5 || mw == 7) && al(img, 4LL * pitch) && al(out, 4LL * out_pitch) &&
+           w % 4 == 0 && w >= 8 && h >= 8;
+}
+
+// Does the launch give every SM a CTA (ngx x bands >= SMs)?  AUTO takes the band kernel only
+// then: on narrower images the TMA-staged / streaming kernels measured faster (512^2).
+bool ispi_sep_band_fills(int w, int h, int k)
+{
+    const BandGeom g = band_geom(w, h, w, w, ISP_CLAMP, k / 2, SSTRIP, sep_band_blocks_per_sm(k), bands_hint(), 185);
     return (long long)g.ngx * g.nband >= num_sms();
 }
 

@@ -870,6 +870,165 @@ __global__ void __launch_bounds__(NTB, 8) k_sob_band(const __grid_constant__ Sob
     else sob_band_body<false>(p, ring, s * FSTRIP, y0, y1 - y0, lane, cl, cr);
 }
 
+
+// ------------------------------------------------------------------------------ separable u8
+// Separable u8 masks with non-negative integer weights whose products sum to at most the
+// divisor d = 2^s <= 256 (the binomial Gaussians of a7: 3x3 / 16, 5x5 / 256): every
+// horizontal sum and the 2-D sum fit a 16-bit lane, so the Laplace skeleton carries them
+// as pair lanes (E = pixels (0,2), O = (1,3)).  Horizontal K-tap sums by DP4A on byte
+// windows (5 taps: two DP4A, the second with weights (0,0,0,r4) on the next window),
+// vertical K-tap weighted sums over a register ring of K rows, then round-half-up by
+// adding d/2 and taking bits [s, s+8) of each lane (exact: U8Round with a power-of-two
+// divisor; no saturation is needed since the result is <= 255).
+struct SepU8BandParams {
+    BandGeom g;
+    const uint8_t *img;
+    uint8_t *out;
+    uint32_t cword;
+    uint32_t r03, r4w;   // DP4A weight words: (r0, r1, r2, r3) and (0, 0, 0, r4) (K = 3: (r0, r1, r2, 0), 0)
+    int col[5];
+    int shift;           // s: d = 2^s
+};
+
+template <int K, bool CY>
+__device__ __forceinline__ void sepu8_band_body(const SepU8BandParams &p, uint32_t ring, int xs0, int y0, int rows,
+                                                int lane, bool cl, bool cr)
+{
+    constexpr int NW = 2;
+    using B = BandShape<NW>;
+    constexpr int LPX = B::LPX, STRIP = B::STRIP, SLOT = B::SLOT, HY = K / 2;
+    const BandGeom &g = p.g;
+    const int x = xs0 + LPX * lane;
+    const bool active = !cr || x < g.w;
+    const bool redge = cr && x + LPX == g.w;
+    const int nin = rows + 2 * HY;
+    const uint32_t loff = LPX * lane;
+    int acol = xs0 - 4, bcol = xs0 + STRIP;
+    uint32_t aon = lane == 0 && (!cl || g.mode == ISP_REPEAT), bdst = 16 + STRIP, bon = !cr && lane == 31;
+    if (cl) acol = g.w - 4;
+    if (redge && g.mode == ISP_REPEAT) { bon = 1; bcol = 0; bdst = 16 + LPX * (lane + 1); }
+    uint32_t sl_ = 0x3210, sr_ = 0x3210;
+    if (cl && lane == 0) sl_ = g.mode == ISP_CLAMP ? 0x4444 : g.mode == ISP_MIRROR ? 0x4500 : 0x3210;
+    if (redge) sr_ = g.mode == ISP_CLAMP ? 0x7777 : g.mode == ISP_MIRROR ? 0x0067 : 0x3210;
+    if (g.mode == ISP_CONSTANT) {
+        for (int j = 0; j < LR; ++j) {
+            if (cl && lane == 0) sts32(ring + j * SLOT + 12, p.cword);
+            if (redge) sts32(ring + j * SLOT + 16 + LPX * (lane + 1), p.cword);
+        }
+    }
+    const int mcol = active ? x : 0;
+    const uint8_t *nrp = p.img + (ptrdiff_t)(y0 - HY) * g.pitch;
+    auto issue = [&](int j, uint32_t slot) {
+        const uint8_t *rp = nrp;
+        if constexpr (CY) {
+            const int yy = map_row1<true>(y0 - HY + j, g.h, g.mode);
+            if (yy < 0) {
+#pragma unroll
+                for (int q = 0; q < NW; ++q) sts32(slot + 16 + loff + 4 * q, p.cword);
+                if (lane == 0) sts32(slot + 12, p.cword);
+                if (lane == 31) sts32(slot + 16 + STRIP, p.cword);
+                return;
+            }
+            rp = p.img + (size_t)yy * g.pitch;
+        }
+        cpa_own<NW>(slot + 16 + loff, rp + mcol, active);
+        cpa4p(slot + 12, rp + acol, aon);
+        cpa4p(slot + bdst, rp + bcol, bon);
+    };
+#pragma unroll
+    for (int j = 0; j < LD; ++j) {
+        issue(j, ring + j * SLOT);
+        nrp += g.pitch;
+        cpa_commit();
+    }
+    const uint32_t halfw = 0x00010001u * (uint32_t)((1 << p.shift) >> 1);
+    uint32_t hr[K][2 * NW];   // horizontal sums of the last K rows as pair lanes (E0, O0, E1, O1)
+    uint8_t *orow = p.out + (ptrdiff_t)(y0 - (K - 1)) * g.out_pitch + x;
+#pragma unroll 1
+    for (int i0 = 0; i0 < nin; i0 += K) {
+#pragma unroll
+        for (int k = 0; k < K; ++k) {
+            const int i = i0 + k;
+            if (i < nin) {
+                cpa_wait<LD - 1>();
+                __syncwarp();
+                const uint32_t sl = ring + (i & (LR - 1)) * SLOT + loff;
+                uint32_t W[NW + 2];
+                lds_own<NW>(sl + 16, *reinterpret_cast<uint32_t(*)[NW]>(&W[1]));
+                W[0] = __byte_perm(lds32(sl + 12), W[1], sl_);
+                W[NW + 1] = __byte_perm(lds32(sl + 16 + LPX), W[NW], sr_);
+                // byte windows F[j] = bytes j-2 .. j+1 relative to the lane's pixel 0, j = 0..8
+                uint32_t F[9];
+#pragma unroll
+                for (int j = 0; j < 9; ++j) {
+                    const int q = (j + 2) >> 2, sh = (j + 2) & 3;   // window starts in word q-1 ... of W (offset -4)
+                    F[j] = sh == 0 ? W[q] : __funnelshift_r(W[q], W[q + 1], 8 * sh);
+                }
+                uint32_t H[8];
+#pragma unroll
+                for (int px = 0; px < 8; ++px) {
+                    if constexpr (K == 5) H[px] = __dp4a(F[px + 1], p.r4w, __dp4a(F[px], p.r03, 0u));   // bytes px-2..px+2
+                    else H[px] = __dp4a(F[px + 1], p.r03, 0u);                                        // bytes px-1..px+1
+                }
+                uint32_t(&hn)[2 * NW] = hr[k];
+                hn[0] = H[2] * 65536u + H[0];
+                hn[1] = H[3] * 65536u + H[1];
+                hn[2] = H[6] * 65536u + H[4];
+                hn[3] = H[7] * 65536u + H[5];
+                if (i >= K - 1 && active) {
+                    // output row y0 + i - (K-1): rows i-K+1 .. i = ring slots (k+1+j) % K
+                    uint32_t v[2 * NW];
+#pragma unroll
+                    for (int q = 0; q < 2 * NW; ++q) {
+                        uint32_t a = halfw;
+#pragma unroll
+                        for (int j = 0; j < K; ++j) a += (uint32_t)p.col[j] * hr[(k + 1 + j) % K][q];
+                        v[q] = (a >> p.shift) & 0x00FF00FFu;
+                    }
+                    *reinterpret_cast<uint2 *>(orow) = make_uint2(__byte_perm(v[0], v[1], 0x6240), __byte_perm(v[2], v[3], 0x6240));
+                }
+                orow += g.out_pitch;
+                if (i + LD < nin) issue(i + LD, ring + ((i + LD) & (LR - 1)) * SLOT);
+                nrp += g.pitch;
+                cpa_commit();
+            }
+        }
+    }
+}
+
+template <int K>
+__global__ void __launch_bounds__(NTB, 8) k_sepu8_band(const __grid_constant__ SepU8BandParams p)
+{
+    __shared__ __align__(16) uint8_t rings[BW][LR * BandShape<2>::SLOT];
+    asm volatile("griddepcontrol.wait;" ::: "memory");
+    asm volatile("griddepcontrol.launch_dependents;");
+    const BandGeom &g = p.g;
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int gx = (int)blockIdx.x % g.ngx, band = (int)blockIdx.x / g.ngx;
+    const int s = gx * BW + warp;
+    if (s >= g.nstrip) return;
+    int y0, y1;
+    band_rows(band, g.nband, g.h, y0, y1);
+    const bool cl = s < g.sx0, cr = s >= g.sx1, cy = band < g.by0 || band >= g.by1;
+    const uint32_t ring = su32(rings[warp]);
+    if (cy) sepu8_band_body<K, true>(p, ring, s * BandShape<2>::STRIP, y0, y1 - y0, lane, cl, cr);
+    else sepu8_band_body<K, false>(p, ring, s * BandShape<2>::STRIP, y0, y1 - y0, lane, cl, cr);
+}
+
+int sepu8_blocks_per_sm(int k)
+{
+    static int nb[2] = {-1, -1};
+    int &v = nb[k == 5];
+    if (v < 0) {
+        const void *fn = k == 5 ? (const void *)k_sepu8_band<5> : (const void *)k_sepu8_band<3>;
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&v, fn, NTB, 0) != cudaSuccess) {
+            cudaGetLastError();
+            v = 0;
+        }
+    }
+    return v;
+}
+
 // Words per lane of the Laplace band launch: 4 (16 pixels) unless ISP_BAND_NW=2
 int band_nw()
 {
@@ -1019,4 +1178,53 @@ cudaError_t ispi_sobel_band(const uint8_t *img, int w, int h, int pitch, int mod
     p.cword = 0x01010101u * (uint32_t)(cval & 0xff);
     bounds[0] = p.g.sx0; bounds[1] = std::max(p.g.sx0, p.g.sx1); bounds[2] = p.g.by0; bounds[3] = p.g.by1;
     return launch_band((const void *)k_sob_band, &p, p.g.ngx * p.g.nband, st);
+}
+
+// Separable u8 band kernel eligibility: K = 3 / 5, non-negative weights, divisor 2^s <= 256
+// with sum(row) * sum(col) <= divisor (16-bit lanes, no saturation), 8-pixel lane granules,
+// 8-byte aligned rows, h >= 8.
+bool ispi_sepu8_band_ok(const void *img, int w, int h, int pitch, const void *out, int out_pitch, int k,
+                        const int *row, const int *col, int divisor)
+{
+    auto al = [](const void *q, long long pb, int a) { return ((uintptr_t)q % a) == 0 && (pb % a) == 0; };
+    if ((k != 3 && k != 5) || divisor <= 0 || divisor > 256 || (divisor & (divisor - 1)) != 0) return false;
+    long long sr = 0, sc = 0;
+    for (int i = 0; i < k; ++i) {
+        if (row[i] < 0 || col[i] < 0 || row[i] > 255) return false;
+        sr += row[i];
+        sc += col[i];
+    }
+    return sr * sc <= divisor && al(img, pitch, 8) && al(out, out_pitch, 8) && w % 8 == 0 && w >= 16 && h >= 8;
+}
+
+void ispi_sepu8_band_shape(int w, int h, int k, int *tw, int *th)
+{
+    const BandGeom g = band_geom(w, h, w, w, ISP_CLAMP, k / 2, 256, sepu8_blocks_per_sm(k), bands_hint());
+    *tw = 256;
+    *th = (h + g.nband - 1) / g.nband;
+}
+
+int ispi_sepu8_band_blocks_per_sm(int k) { return sepu8_blocks_per_sm(k); }
+
+cudaError_t ispi_sepu8_band(const uint8_t *img, int w, int h, int pitch, int k, const int *row, const int *col,
+                            int divisor, int mode, int cval, uint8_t *out, int out_pitch, cudaStream_t st, int bounds[4])
+{
+    SepU8BandParams p{};
+    p.g = band_geom(w, h, pitch, out_pitch, mode, k / 2, 256, sepu8_blocks_per_sm(k), bands_hint());
+    p.img = img;
+    p.out = out;
+    p.cword = 0x01010101u * (uint32_t)(cval & 0xff);
+    if (k == 5) {
+        p.r03 = (uint32_t)row[0] | (uint32_t)row[1] << 8 | (uint32_t)row[2] << 16 | (uint32_t)row[3] << 24;
+        p.r4w = (uint32_t)row[4] << 24;
+    } else {
+        p.r03 = (uint32_t)row[0] | (uint32_t)row[1] << 8 | (uint32_t)row[2] << 16;
+        p.r4w = 0;
+    }
+    for (int j = 0; j < k; ++j) p.col[j] = col[j];
+    int s = 0;
+    while ((1 << s) < divisor) ++s;
+    p.shift = s;
+    bounds[0] = p.g.sx0; bounds[1] = std::max(p.g.sx0, p.g.sx1); bounds[2] = p.g.by0; bounds[3] = p.g.by1;
+    return launch_band(k == 5 ? (const void *)k_sepu8_band<5> : (const void *)k_sepu8_band<3>, &p, p.g.ngx * p.g.nband, st);
 }

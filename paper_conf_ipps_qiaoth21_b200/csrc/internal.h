@@ -52,6 +52,7 @@ cudaError_t ispi_fused_band(const uint8_t *img, int w, int h, int pitch, int mod
                             cudaStream_t st);
 // separable f32 band kernel (band_f32.cu): ISP_TMA / AUTO of whole-image separable f32 masks
 int ispi_sep_band_blocks_per_sm(int k);
+bool ispi_sep_band_fills(int w, int h, int k);
 bool ispi_sep_band_ok(const float *img, int w, int h, int pitch, const float *out, int out_pitch, int mw, int mh);
 void ispi_sep_band_shape(int w, int h, int k, int *tw, int *th);
 cudaError_t ispi_sep_band(const float *img, int w, int h, int pitch, const float *row, const float *col, int k,
@@ -61,3 +62,9 @@ bool ispi_band_sobel_ok(const void *img, int w, int h, int pitch, const void *dx
 void ispi_band_sobel_shape(int w, int h, int *tw, int *th);
 cudaError_t ispi_sobel_band(const uint8_t *img, int w, int h, int pitch, int mode, int cval, int16_t *dx, int16_t *dy,
                             uint8_t *mag, int out_pitch, cudaStream_t st, int bounds[4]);
+bool ispi_sepu8_band_ok(const void *img, int w, int h, int pitch, const void *out, int out_pitch, int k,
+                        const int *row, const int *col, int divisor);
+void ispi_sepu8_band_shape(int w, int h, int k, int *tw, int *th);
+int ispi_sepu8_band_blocks_per_sm(int k);
+cudaError_t ispi_sepu8_band(const uint8_t *img, int w, int h, int pitch, int k, const int *row, const int *col,
+                            int divisor, int mode, int cval, uint8_t *out, int out_pitch, cudaStream_t st, int bounds[4]);
