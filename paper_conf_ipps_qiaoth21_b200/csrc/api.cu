@@ -579,7 +579,7 @@ isp_status_t resolve_and_launch(Desc &d, int fam, int w, int h, int mw, int mh, 
         info.o_naive = nb_naive > 0 ? occupancy_of(nb_naive, threads) : 1.0;
         // staged / tiled kernels (TMA): latency is hidden by the staging, not by resident
         // warps, so their occupancy term is the naive kernel's (reading A34)
-        info.o_isp = chosen == ISP_TMA ? info.o_naive
+        info.o_isp = chosen == ISP_TMA ? info.o_naive * std::min(1.0, (double)p.nx * p.ny / num_sms())
                                        : (nb_stream > 0 ? occupancy_of(nb_stream, threads) : 1.0);
         n_block(p, info.n_block);
         if (chosen == ISP_TMA) mp.form = 2;   // staged kernels: checks per staged element (A21)
@@ -688,7 +688,9 @@ bool tile_variant(int which, int fam, int mode, int w, int h, int mw, int mh, is
                        : which >= 2 ? ispi_band_blocks_per_sm(which == 3 ? 1 : 0)
                                     : ispi_tile_blocks_per_sm(which);
         info.o_naive = 0.5;   // the naive streaming kernel (64 regs x 128 threads: 8 blocks / SM)
-        info.o_isp = which >= 2 ? info.o_naive : occupancy_of(nb > 0 ? nb : 1, 128);
+        // band kernels (A34): the naive kernel's occupancy on the SMs the launch reaches
+        const double reach = std::min(1.0, (double)ceil_div(p.nx, 4) * p.ny / num_sms());
+        info.o_isp = which >= 2 ? info.o_naive * reach : occupancy_of(nb > 0 ? nb : 1, 128);
         model(p, w, h, mw, mh, mp, info);
         if (which >= 2 && p.degenerate) {
             // a band kernel runs one-strip / one-band images too (its edge warps check both
@@ -967,8 +969,7 @@ isp_status_t ispi_filter_f32(const float *img, int w, int h, int pitch, const fl
             isp_status_t ts;
             if (!rr && !getenv("ISP_F32_STAGED") &&
                 tile_variant(4, F_SEP_F32, border_mode, w, h, mw, mh, variant,
-                             ispi_sep_band_ok(img, w, h, pitch, out, out_pitch, mw, mh) &&
-                                 (variant == ISP_TMA || ispi_sep_band_fills(w, h, mw)),
+                             ispi_sep_band_ok(img, w, h, pitch, out, out_pitch, mw, mh),
                              [&](int *b) { return ispi_sep_band(img, w, h, pitch, row.data(), col.data(), mw,
                                                                border_mode, const_val, out, out_pitch,
                                                                (cudaStream_t)stream, b); },

@@ -261,13 +261,6 @@ bool ispi_sep_band_ok(const float *img, int w, int h, int pitch, const float *ou
            w % 4 == 0 && w >= 8 && h >= 8;
 }
 
-// Does the launch give every SM a CTA (ngx x bands >= SMs)?  AUTO takes the band kernel only
-// then: on narrower images the TMA-staged / streaming kernels measured faster (512^2).
-bool ispi_sep_band_fills(int w, int h, int k)
-{
-    const BandGeom g = band_geom(w, h, w, w, ISP_CLAMP, k / 2, SSTRIP, sep_band_blocks_per_sm(k), bands_hint(), 185);
-    return (long long)g.ngx * g.nband >= num_sms();
-}
 
 void ispi_sep_band_shape(int w, int h, int k, int *tw, int *th)
 {

@@ -52,7 +52,6 @@ cudaError_t ispi_fused_band(const uint8_t *img, int w, int h, int pitch, int mod
                             cudaStream_t st);
 // separable f32 band kernel (band_f32.cu): ISP_TMA / AUTO of whole-image separable f32 masks
 int ispi_sep_band_blocks_per_sm(int k);
-bool ispi_sep_band_fills(int w, int h, int k);
 bool ispi_sep_band_ok(const float *img, int w, int h, int pitch, const float *out, int out_pitch, int mw, int mh);
 void ispi_sep_band_shape(int w, int h, int k, int *tw, int *th);
 cudaError_t ispi_sep_band(const float *img, int w, int h, int pitch, const float *row, const float *col, int k,
