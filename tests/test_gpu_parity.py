@@ -306,20 +306,22 @@ def test_cfg5_gauss7_f32_16384_single_gpu(isp):
     n = 16384
     g = torch.Generator(device="cuda").manual_seed(5)
     d = torch.rand((n, n), device="cuda", generator=g)
-    rows = sample_rows(n, k=8, seed=5)
+    # sampled rows plus the image's first / last three (the T / B regions of every kernel)
+    rows = sorted(set(sample_rows(n, k=8, seed=5)) | {0, 1, 2, n - 3, n - 2, n - 1})
     band = sorted(set(r + k for r in rows for k in range(-3, 4) if 0 <= r + k < n) | {0, 1, 2, n - 3, n - 2, n - 1})
     mask = binomial_f32(7)
-    for mode in ["clamp", "repeat"]:
-        got = isp.isp_filter(d, mask, mode)
+    cval = 0.25
+    for mode in MODES:
+        got = isp.isp_filter(d, mask, mode, cval)
         # oracle on the rows the sampled outputs depend on (plus the border rows the maps reach)
         sub = d[band].cpu().numpy()
         ref_full_rows = []
         for r in rows:
-            ys = [oracle.border_index(mode, r + k, n) for k in range(-3, 4)]
-            win = np.stack([sub[band.index(y)] for y in ys])
-            # rows of `win` are already the mapped y taps: row 3's output uses exactly them;
-            # x is handled by the oracle's own border map
-            out, sc = oracle.filter_f64(win, mask, mode, rows=(3, 4), with_scale=True)
+            ys = [oracle.border_index(mode, r + k, n) if mode != "constant" else r + k for k in range(-3, 4)]
+            win = np.stack([sub[band.index(y)] if 0 <= y < n else np.full(n, cval, dtype=np.float32) for y in ys])
+            # rows of `win` are already the mapped y taps (Constant: rows of C): row 3's output
+            # uses exactly them; x is handled by the oracle's own border map
+            out, sc = oracle.filter_f64(win, mask, mode, cval, rows=(3, 4), with_scale=True)
             ref_full_rows.append((out[0], sc[0]))
         ref = np.stack([r for r, _ in ref_full_rows])
         sc = np.stack([s for _, s in ref_full_rows])
