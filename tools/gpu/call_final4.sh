@@ -1,0 +1,16 @@
+# Final measurement of the committed band-kernel build (one gpurun call).
+set -x
+md5sum paper_conf_ipps_qiaoth21_b200/libisp.so
+python -c "import __graft_entry__ as g; g.smoke()" 2>&1 | tail -1
+timeout 1500 python -m pytest tests -m gpu -q -p no:cacheprovider 2>&1 | grep -v "^E   *\[" | tail -4
+timeout 900 python bench.py --steps 20 --warmup 5 > gpurun_out/r03_bench.json 2> gpurun_out/r03_bench.err
+timeout 900 python bench.py --workload cfg5 --steps 20 --warmup 5 > gpurun_out/r03_bench_cfg5.json 2> gpurun_out/r03_bench_cfg5.err
+timeout 600 python bench.py --impl reference --steps 3 --warmup 3 > gpurun_out/r03_ref.json 2>&1
+timeout 900 python tools/ncu_counters.py --tag r03 --out-dir gpurun_out > gpurun_out/r03_counters.log 2>&1; tail -2 gpurun_out/r03_counters.log
+timeout 600 python tools/bench_suite.py > gpurun_out/r03_suite.json 2> gpurun_out/r03_suite.err
+for m in mirror clamp repeat constant; do timeout 300 python tools/fused_time.py --mode $m 2>&1 | tail -1; done > gpurun_out/r03_fused.jsonl
+timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --csv --log-file gpurun_out/r03_launches.csv python bench.py --steps 2 --warmup 3 --quick --no-cpu > /dev/null 2>&1
+python -c "
+import json
+for f in ['gpurun_out/r03_bench.json','gpurun_out/r03_bench_cfg5.json']:
+    d=json.loads(open(f).read().strip().splitlines()[-1]); print(f, d['value'], d['roofline']['frac'], d['roofline']['duration_us'], d['clocks'])"

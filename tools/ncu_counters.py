@@ -78,6 +78,8 @@ def cases():
                         lambda m=mode, v=v: isp.isp_atrous_f32(f, 2, m, 0.5, out=fo, variant=v)))
             out.append((f"bilateral13_f32/{mode}/{v}", "bilateral", 13, 13, px2,
                         lambda m=mode, v=v: isp.isp_bilateral_f32(fb, 13, 3.0, 0.1, m, 0.5, out=fbo, variant=v)))
+        out.append((f"gauss5_u8/{mode}/tma", "u8", 5, 5, px4,
+                    lambda m=mode: isp.isp_filter_u8(u8, G5, int(G5.sum()), m, 7, out=u8o, variant="tma")))
         out.append((f"bilateral13_f32/{mode}/tma", "bilateral", 13, 13, px2,
                     lambda m=mode: isp.isp_bilateral_f32(fb, 13, 3.0, 0.1, m, 0.5, out=fbo, variant="tma")))
     for v in ["tma", "warp", "naive"]:
@@ -139,7 +141,7 @@ def markdown(out, tag):
 
 def main():
     ap = argparse.ArgumentParser()
-    ap.add_argument("--tag", default="r02")
+    ap.add_argument("--tag", default="r03")
     ap.add_argument("--out-dir", default=os.path.join(ROOT, "profiles"))
     ap.add_argument("--inner", action="store_true")
     ap.add_argument("--labels", default="/tmp/ncu_counter_labels.json")
