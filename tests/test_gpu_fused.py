@@ -110,13 +110,16 @@ def test_fused_cfg3_4096(isp):
     np.testing.assert_array_equal(host(har)[rows], oracle.harris(rdx, rdy, "mirror", rows=rows))
 
 
+@pytest.mark.parametrize("variant", ["tma", "warp"])
 @pytest.mark.parametrize("shape", [(70, 2064), (100, 1040), (66, 272), (129, 4112)])
 @pytest.mark.parametrize("kind", ["structured", "noise"])
-def test_fused_tile_isp_kernel(isp, shape, kind):
-    """The tile-ISP kernel (k_fused_body: Body tiles unchecked, border tiles staged through
-    the pattern with the ext fix-up at remapped coordinates) on aligned images with partial
-    right / bottom tiles: every output bit-exact against the oracle composition, all
-    modes, several thresholds (the f32 Harris path with its exact f64 fallback)."""
+def test_fused_tile_isp_kernel(isp, shape, kind, variant):
+    """The band kernel (tma: k_fused_band, remapped Harris ext by edge-lane permutes and ring
+    copies) and the tile-ISP kernel (warp: k_fused_body, Body tiles unchecked, border tiles
+    staged through the pattern with the ext fix-up at remapped coordinates) on aligned
+    images with partial right / bottom strips and tiles: every output bit-exact against the
+    oracle composition, all modes, several thresholds (the f32 Harris path with its exact
+    f64 fallback)."""
     h, w = shape
     img = synth.structured_u8(h, w, 8) if kind == "structured" else synth.uniform_u8(h, w, 8)
     d = dev(img)
@@ -126,7 +129,47 @@ def test_fused_tile_isp_kernel(isp, shape, kind):
             rdx, rdy, rmag, rlap, rhar = composition(img, mode, 17, hc, thr)
             dx = torch.empty((h, w), dtype=torch.int16, device="cuda")
             dy = torch.empty_like(dx)
-            mag, lap, har = isp.isp_pipeline_cfg3_u8(d, mode, 17, hc, thr, dx=dx, dy=dy)
+            mag, lap, har = isp.isp_pipeline_cfg3_u8(d, mode, 17, hc, thr, dx=dx, dy=dy, variant=variant)
             for name, got, ref in [("dx", dx, rdx), ("dy", dy, rdy), ("mag", mag, rmag), ("lap", lap, rlap),
                                    ("harris", har, rhar)]:
                 np.testing.assert_array_equal(host(got), ref, err_msg=f"{name} {mode} {thr} {shape} {kind}")
+
+
+def _r25(dx, dy, mode, c, y, x):
+    """Exact R25 at (y, x) in Python integers, the dx / dy IMAGES read through the oracle's
+    border map (Constant: the Harris constant outside)."""
+    h, w = dx.shape
+    wts = [1, 2, 1]
+    sxx = syy = sxy = 0
+    for j in range(3):
+        for i in range(3):
+            yy, xx = oracle.border_index(mode, y + j - 1, h), oracle.border_index(mode, x + i - 1, w)
+            gx, gy = (c, c) if (yy < 0 or xx < 0) else (int(dx[yy, xx]), int(dy[yy, xx]))
+            sxx += wts[j] * wts[i] * gx * gx
+            syy += wts[j] * wts[i] * gy * gy
+            sxy += wts[j] * wts[i] * gx * gy
+    return 25 * (sxx * syy - sxy * sxy) - (sxx + syy) ** 2
+
+
+def test_fused_band_pitched_and_threshold_boundary(isp):
+    """The band kernel on a pitched image (w = 336 of a 352-byte pitch, outputs pitched too)
+    and Harris thresholds at R-1, R, R+1 of chosen pixels (including border ones whose
+    window reads remapped dx / dy): exact decisions and nothing written past the width."""
+    h, w, pitch = 61, 336, 352
+    img = synth.uniform_u8(h, w, 19)
+    d = dev(synth.pitched(img, pitch, 99))
+    for mode in MODES:
+        hc = 1020 if mode == "constant" else 0
+        rdx, rdy, rmag, rlap, _ = composition(img, mode, 5, hc, 0)
+        for (y, x) in [(0, 0), (h - 1, w - 1), (30, 170), (1, w - 2)]:
+            R = _r25(rdx, rdy, mode, hc, y, x)
+            for thr in (R - 1, R, R + 1):
+                mag = torch.zeros((h, pitch), dtype=torch.uint8, device="cuda")
+                lap, har = torch.zeros_like(mag), torch.zeros_like(mag)
+                isp.isp_pipeline_cfg3_u8(d, mode, 5, hc, thr, mag=mag, lap=lap, harris=har, w=w, variant="tma")
+                ref = oracle.harris(rdx, rdy, mode, hc, thr)
+                np.testing.assert_array_equal(host(har)[:, :w], ref, err_msg=f"harris {mode} thr={thr}")
+                assert host(har)[y, x] == (255 if R > thr else 0)
+                np.testing.assert_array_equal(host(mag)[:, :w], rmag, err_msg=f"mag {mode}")
+                np.testing.assert_array_equal(host(lap)[:, :w], rlap, err_msg=f"lap {mode}")
+                assert not host(mag)[:, w:].any() and not host(har)[:, w:].any()
