@@ -273,50 +273,28 @@ constexpr int HLD = 5;                      // rows in flight per warp
 
 struct HRow { float2 xxE, xxO, yyE, yyO, xyE, xyO; };
 
-// int16 halves of words as exact floats: w ^ 0x80008000 holds v + 32768 in each half, which
-// a byte permute places in the mantissa of 2^23 (bits 0x4B00xxxx); one packed subtract of
-// 2^23 + 32768 then yields the pair exactly.  lo: the low halves of (a, b), hi: the high.
-__device__ __forceinline__ float2 lo2(uint32_t a, uint32_t b)
+// int16 halves (sa of a, sb of b: 0x7610 = low half, 0x7632 = high half) as an exact float
+// pair: the biased halves land in the mantissa of 2^23, one packed subtract removes 2^23 + 32768
+__device__ __forceinline__ float2 i16pair(uint32_t a, uint32_t sa, uint32_t b, uint32_t sb)
 {
-    const float2 r = make_float2(__uint_as_float(__byte_perm(a ^ 0x80008000u, 0x4B000000u, 0x7610)),
-                                 __uint_as_float(__byte_perm(b ^ 0x80008000u, 0x4B000000u, 0x7610)));
-    return add2(r, f2(-8421376.0f, -8421376.0f));
-}
-__device__ __forceinline__ float2 hi2(uint32_t a, uint32_t b)
-{
-    const float2 r = make_float2(__uint_as_float(__byte_perm(a ^ 0x80008000u, 0x4B000000u, 0x7632)),
-                                 __uint_as_float(__byte_perm(b ^ 0x80008000u, 0x4B000000u, 0x7632)));
+    const float2 r = make_float2(__uint_as_float(__byte_perm(a ^ 0x80008000u, 0x4B000000u, sa)),
+                                 __uint_as_float(__byte_perm(b ^ 0x80008000u, 0x4B000000u, sb)));
     return add2(r, f2(-8421376.0f, -8421376.0f));
 }
 
 // Horizontal [1,2,1] sums of xx, yy, xy for pixels 0..3 from the words (L, X0, X1, R) of dx
-// and dy (L = pixels -2,-1; R = 4,5).  Products of integers <= 1020 are exact in f32.
+// and dy (L = pixels -2,-1; R = 4,5) through the pairs A = (p-1, p1), E, O, B = (p2, p4)
+// (har_hrow_f: no pair shuffling).  Products of integers <= 1020 are exact in f32.
+__device__ __forceinline__ HRow har_hrow_f(float2 xA, float2 xE, float2 xO, float2 xB, float2 yA, float2 yE, float2 yO,
+                                           float2 yB);
 __device__ __forceinline__ HRow har_hrow(uint32_t XL, uint32_t X0, uint32_t X1, uint32_t XR, uint32_t YL, uint32_t Y0,
                                          uint32_t Y1, uint32_t YR)
 {
-    const float2 xE = lo2(X0, X1), xO = hi2(X0, X1), yE = lo2(Y0, Y1), yO = hi2(Y0, Y1);
-    // edge pixels p-1 (high half of L) and p4 (low half of R) as pairs (p-1, p4)
-    const float2 xe = add2(make_float2(__uint_as_float(__byte_perm(XL ^ 0x80008000u, 0x4B000000u, 0x7632)),
-                                       __uint_as_float(__byte_perm(XR ^ 0x80008000u, 0x4B000000u, 0x7610))),
-                           f2(-8421376.0f, -8421376.0f));
-    const float2 ye = add2(make_float2(__uint_as_float(__byte_perm(YL ^ 0x80008000u, 0x4B000000u, 0x7632)),
-                                       __uint_as_float(__byte_perm(YR ^ 0x80008000u, 0x4B000000u, 0x7610))),
-                           f2(-8421376.0f, -8421376.0f));
-    const float2 xxE = mul2(xE, xE), xxO = mul2(xO, xO), yyE = mul2(yE, yE), yyO = mul2(yO, yO);
-    const float2 xyE = mul2(xE, yE), xyO = mul2(xO, yO);
-    const float2 xxe = mul2(xe, xe), yye = mul2(ye, ye), xye = mul2(xe, ye);
-    const float2 xxA = f2(xxe.x, xxO.x), xxB = f2(xxE.y, xxe.y);
-    const float2 yyA = f2(yye.x, yyO.x), yyB = f2(yyE.y, yye.y);
-    const float2 xyA = f2(xye.x, xyO.x), xyB = f2(xyE.y, xye.y);
-    const float2 two = f2(2.f, 2.f);
-    HRow h;
-    h.xxE = add2(fma2(two, xxE, xxA), xxO);   // (H0, H2) = A + 2E + O, A = (p-1, p1)
-    h.xxO = add2(fma2(two, xxO, xxE), xxB);   // (H1, H3) = E + 2O + B, B = (p2, p4)
-    h.yyE = add2(fma2(two, yyE, yyA), yyO);
-    h.yyO = add2(fma2(two, yyO, yyE), yyB);
-    h.xyE = add2(fma2(two, xyE, xyA), xyO);
-    h.xyO = add2(fma2(two, xyO, xyE), xyB);
-    return h;
+    const float2 xA = i16pair(XL, 0x7632, X0, 0x7632), xE = i16pair(X0, 0x7610, X1, 0x7610);
+    const float2 xO = i16pair(X0, 0x7632, X1, 0x7632), xB = i16pair(X1, 0x7610, XR, 0x7610);
+    const float2 yA = i16pair(YL, 0x7632, Y0, 0x7632), yE = i16pair(Y0, 0x7610, Y1, 0x7610);
+    const float2 yO = i16pair(Y0, 0x7632, Y1, 0x7632), yB = i16pair(Y1, 0x7610, YR, 0x7610);
+    return har_hrow_f(xA, xE, xO, xB, yA, yE, yO, yB);
 }
 
 // R25 > thr for a pixel pair, exact (reading A33).  f32 evaluation
