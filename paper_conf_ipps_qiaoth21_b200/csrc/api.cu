@@ -965,14 +965,14 @@ isp_status_t ispi_filter_f32(const float *img, int w, int h, int pitch, const fl
         if (separable_f32(mask, mw, mh, row, col)) {
             d.rowf = row.data();
             d.colf = col.data();
-            // ISP_TMA / AUTO on whole images: the warp-strip band kernel (band_f32.cu)
+            // ISP_TMA / AUTO: the warp-strip band kernel (band_f32.cu; whole images and strips)
             isp_status_t ts;
-            if (!rr && !getenv("ISP_F32_STAGED") &&
-                tile_variant(4, F_SEP_F32, border_mode, w, h, mw, mh, variant,
-                             ispi_sep_band_ok(img, w, h, pitch, out, out_pitch, mw, mh),
+            if (!getenv("ISP_F32_STAGED") &&
+                tile_variant(4, F_SEP_F32, border_mode, w, rr ? rr->nrows : h, mw, mh, variant,
+                             ispi_sep_band_ok(img, w, rr ? rr->nrows : h, pitch, out, out_pitch, mw, mh),
                              [&](int *b) { return ispi_sep_band(img, w, h, pitch, row.data(), col.data(), mw,
                                                                border_mode, const_val, out, out_pitch,
-                                                               (cudaStream_t)stream, b); },
+                                                               (cudaStream_t)stream, b, rr); },
                              ts, "isp_filter(separable band)"))
                 return ts;
             return resolve_and_launch(d, F_SEP_F32, w, h, mw, mh, mw / 2, mh / 2, false, variant, kfn_sep_f32,

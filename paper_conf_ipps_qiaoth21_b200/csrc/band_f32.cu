@@ -37,8 +37,19 @@ constexpr int SLD = BAND_F32_D;
 #endif
 static_assert(LR >= SLD + 1, "ring too small");
 
+// Output rows [oy0, oy0 + nrows) of an image of height g.h (whole image: 0, h); strips of
+// the multi-GPU path (readings A30 / A32): an edge that is not an image edge
+// (t_real / b_real = 0) is a strip edge -- its rows are in the buffer (NCCL halo exchange)
+// or, with peer != 0, in the neighbour strips' buffers peer_lo / peer_hi (global-row
+// addressed, rows < own_y0 / >= own_y1).
+struct SepBandRows {
+    int oy0, nrows, t_real, b_real, peer, own_y0, own_y1;
+    const float *peer_lo, *peer_hi;
+};
+
 struct SepBandParams {
     BandGeom g;
+    SepBandRows rr;
     const float *img;
     float *out;
     float cval;
@@ -108,15 +119,22 @@ __device__ __forceinline__ void sep_band_body(const SepBandParams &p, uint32_t r
     const float *nrp = p.img + (ptrdiff_t)(y0 - HX) * g.pitch;
     auto issue = [&](int j, uint32_t slot) {
         const float *rp = nrp;
-        if constexpr (CY) {
-            const int yy = map_row1<true>(y0 - HX + j, g.h, g.mode);
-            if (yy < 0) {
+        if constexpr (CY) {   // T / B: image edges through the pattern, strip edges by buffer
+            const int y = y0 - HX + j;
+            const bool out_img = (p.rr.t_real && y < 0) || (p.rr.b_real && y >= g.h);
+            const int yy = out_img ? map_row1<true>(y, g.h, g.mode) : y;
+            if (out_img && yy < 0) {   // Constant: the staged row is C
                 sts128f(slot + 16 + loff, p.cval);
                 if (lane == 0) sts128f(slot, p.cval);
                 if (lane == 31) sts128f(slot + 16 + 4 * SSTRIP, p.cval);
                 return;
             }
-            rp = p.img + (size_t)yy * g.pitch;
+            const float *base = p.img;
+            if (p.rr.peer) {
+                if (yy < p.rr.own_y0) base = p.rr.peer_lo;
+                else if (yy >= p.rr.own_y1) base = p.rr.peer_hi;
+            }
+            rp = base + (ptrdiff_t)yy * g.pitch;
         }
         cpa16p(slot + 16 + loff, rp + mcol, active);
         cpa16p(slot, rp + acol, aon);
@@ -129,7 +147,7 @@ __device__ __forceinline__ void sep_band_body(const SepBandParams &p, uint32_t r
         cpa_commit();
     }
     float acc[K][SPX];
-    float *orow = p.out + (ptrdiff_t)(y0 - (K - 1)) * g.out_pitch + x;   // row of output o = r - (K-1)
+    float *orow = p.out + (ptrdiff_t)(y0 - p.rr.oy0 - (K - 1)) * g.out_pitch + x;   // output o = r - (K-1)
 #pragma unroll 1
     for (int r0 = 0; r0 < nin; r0 += K) {
 #pragma unroll
@@ -213,7 +231,9 @@ __global__ void __launch_bounds__(NTB, BAND_F32_MINB) k_sep_band(const __grid_co
     const int s = gx * BW + warp;
     if (s >= g.nstrip) return;
     int y0, y1;
-    band_rows(band, g.nband, g.h, y0, y1);
+    band_rows(band, g.nband, p.rr.nrows, y0, y1);
+    y0 += p.rr.oy0;
+    y1 += p.rr.oy0;
     const bool cl = s < g.sx0, cr = s >= g.sx1, cy = band < g.by0 || band >= g.by1;
     const uint32_t ring = su32(rings[warp]);
     const int xs0 = s * SSTRIP, rows = y1 - y0;
@@ -270,10 +290,33 @@ void ispi_sep_band_shape(int w, int h, int k, int *tw, int *th)
 }
 
 cudaError_t ispi_sep_band(const float *img, int w, int h, int pitch, const float *row, const float *col, int k,
-                          int mode, float cval, float *out, int out_pitch, cudaStream_t st, int bounds[4])
+                          int mode, float cval, float *out, int out_pitch, cudaStream_t st, int bounds[4],
+                          const RowRange *rr)
 {
     SepBandParams p{};
-    p.g = band_geom(w, h, pitch, out_pitch, mode, k / 2, SSTRIP, sep_band_blocks_per_sm(k), bands_hint(), 185);
+    const int nrows = rr ? rr->nrows : h;
+    p.g = band_geom(w, nrows, pitch, out_pitch, mode, k / 2, SSTRIP, sep_band_blocks_per_sm(k), bands_hint(), 185);
+    p.g.h = h;
+    p.rr = SepBandRows{0, h, 1, 1, 0, 0, h, nullptr, nullptr};
+    if (rr) {
+        p.rr = SepBandRows{rr->oy0, rr->nrows, rr->t_real, rr->b_real, rr->peer, rr->own_y0, rr->own_y1,
+                           static_cast<const float *>(rr->peer_lo), static_cast<const float *>(rr->peer_hi)};
+        // bands needing the T / B body: image edges are mapped, strip edges of the peer path
+        // read the neighbours' buffers; a strip edge of the NCCL path reads its own halo rows
+        const int hy = k / 2;
+        auto top = [&](int b) {
+            const int y0 = rr->oy0 + (int)((long long)b * nrows / p.g.nband);
+            return (rr->t_real && y0 - hy < 0) || (rr->peer && y0 - hy < rr->own_y0);
+        };
+        auto bot = [&](int b) {
+            const int y1 = rr->oy0 + (int)((long long)(b + 1) * nrows / p.g.nband);
+            return (rr->b_real && y1 + hy > h) || (rr->peer && y1 + hy > rr->own_y1);
+        };
+        p.g.by0 = 0;
+        while (p.g.by0 < p.g.nband && top(p.g.by0)) ++p.g.by0;
+        p.g.by1 = p.g.by0;
+        while (p.g.by1 < p.g.nband && !bot(p.g.by1)) ++p.g.by1;
+    }
     p.img = img;
     p.out = out;
     p.cval = cval;

@@ -55,7 +55,8 @@ int ispi_sep_band_blocks_per_sm(int k);
 bool ispi_sep_band_ok(const float *img, int w, int h, int pitch, const float *out, int out_pitch, int mw, int mh);
 void ispi_sep_band_shape(int w, int h, int k, int *tw, int *th);
 cudaError_t ispi_sep_band(const float *img, int w, int h, int pitch, const float *row, const float *col, int k,
-                          int mode, float cval, float *out, int out_pitch, cudaStream_t st, int bounds[4]);
+                          int mode, float cval, float *out, int out_pitch, cudaStream_t st, int bounds[4],
+                          const RowRange *rr = nullptr);
 bool ispi_band_sobel_ok(const void *img, int w, int h, int pitch, const void *dx, const void *dy, const void *mag,
                         int out_pitch);
 void ispi_band_sobel_shape(int w, int h, int *tw, int *th);

@@ -264,15 +264,17 @@ def _strip_run(isp, img, H, W, halo, hy, nranks, r, mode, fill, local_call):
     return y0, sh, local_call(dev(buf))
 
 
+@pytest.mark.parametrize("sep", [False, True])
 @pytest.mark.parametrize("nranks", [2, 3, 5, 8])
 @pytest.mark.parametrize("m", [3, 5, 7, 9])
-def test_strips_isp_f32(isp, nranks, m):
+def test_strips_isp_f32(isp, nranks, m, sep):
     """Strip launches (RowRange, t_real / b_real = 0 at strip edges) of every rank on a
     2052-wide image run non-degenerate ISP bodies and reproduce the single-image result
-    bitwise, with the halo rows filled as the NCCL schedule fills them."""
+    bitwise, with the halo rows filled as the NCCL schedule fills them; separable masks
+    (sep) run the band kernel k_sep_band on the strips (TMA)."""
     H, W = 203, 2052
     img = synth.uniform_f32(H, W, 77)
-    mask = np.random.default_rng(m).random((m, m)).astype(np.float32)
+    mask = binomial_f32(m) if sep else np.random.default_rng(m).random((m, m)).astype(np.float32)
     hy = m // 2
     halo = hy + 1
     full = dev(img)
@@ -431,16 +433,18 @@ def test_sobel_magnitude_near_ties(isp):
 
 
 # ---------------------------------------------------------------- peer-direct strips (N4)
+@pytest.mark.parametrize("sep", [False, True])
 @pytest.mark.parametrize("nranks", [2, 3, 8])
 @pytest.mark.parametrize("m", [3, 7, 9])
-def test_peer_strips_f32(isp, nranks, m):
+def test_peer_strips_f32(isp, nranks, m, sep):
     """Peer-direct strips: every rank's buffer holds only its own rows,
     the neighbour rows are read from the neighbours' buffers (separate allocations, as
     IPC mappings would be), ONE launch per rank; the gathered result equals the
-    single-image result bitwise, strip-edge block rows run T / B bodies (non-degenerate)."""
+    single-image result bitwise, strip-edge block rows run T / B bodies (non-degenerate);
+    separable masks (sep) run the band kernel, whose strip-edge bands select the buffer."""
     H, W = 203, 2052
     img = synth.uniform_f32(H, W, 79)
-    mask = np.random.default_rng(m).random((m, m)).astype(np.float32)
+    mask = binomial_f32(m) if sep else np.random.default_rng(m).random((m, m)).astype(np.float32)
     full = dev(img)
     strips = []
     for r in range(nranks):
