@@ -266,9 +266,13 @@ struct HarBandParams {
     float thr_f, thr_err;
 };
 
-constexpr int HSTRIP = 128;                 // columns per warp (4 per lane)
-constexpr int HIMG = 32 + 2 * HSTRIP;       // bytes per image row in a slot: [12,16) left, [16,272) strip, [272,276) right
-constexpr int HSLOT = 2 * HIMG;             // dx row, then dy row
+// G groups of 4 pixels per lane: strips of 128 G columns; a slot holds the dx row then the
+// dy row, each [12,16) left halo word, [16, 16 + 256 G) strip, then the right halo word
+template <int G> struct HarShape {
+    static constexpr int STRIP = 128 * G;
+    static constexpr int IMG = 32 + 2 * STRIP;
+    static constexpr int SLOT = 2 * IMG;
+};
 constexpr int HLD = 5;                      // rows in flight per warp
 
 struct HRow { float2 xxE, xxO, yyE, yyO, xyE, xyO; };
@@ -322,23 +326,24 @@ __device__ __forceinline__ void harris2p(float2 sxx, float2 syy, float2 sxy, flo
     }
 }
 
-template <bool CY>
+template <int G, bool CY>
 __device__ __forceinline__ void har_band_body(const HarBandParams &p, uint32_t ring, int xs0, int y0, int rows,
                                               int lane, bool cl, bool cr)
 {
+    constexpr int STRIP = HarShape<G>::STRIP, HIMG = HarShape<G>::IMG, HSLOT = HarShape<G>::SLOT, NWD = 2 * G;
     const BandGeom &g = p.g;
-    const int x = xs0 + 4 * lane;
+    const int x = xs0 + 4 * G * lane;
     const bool active = !cr || x < g.w;
-    const bool redge = cr && x + 4 == g.w;
+    const bool redge = cr && x + 4 * G == g.w;
     const int nin = rows + 2;   // >= 8
-    const uint32_t loff = 8 * lane;
+    const uint32_t loff = 8 * G * lane;
     // halo copies (columns, in int16 elements): A = lane 0's left word (L, Repeat: w-2, w-1),
     // B = lane 31's right word, or (R, Repeat) the last lane's wrapped word (0, 1)
-    int acol = xs0 - 2, bcol = xs0 + HSTRIP;
-    uint32_t aon = lane == 0 && (!cl || g.mode == ISP_REPEAT), bdst = 16 + 2 * HSTRIP, bon = !cr && lane == 31;
+    int acol = xs0 - 2, bcol = xs0 + STRIP;
+    uint32_t aon = lane == 0 && (!cl || g.mode == ISP_REPEAT), bdst = 16 + 2 * STRIP, bon = !cr && lane == 31;
     if (cl) acol = g.w - 2;
-    if (redge && g.mode == ISP_REPEAT) { bon = 1; bcol = 0; bdst = 16 + 8 * (lane + 1); }
-    // selectors: left word = prmt(loaded, own X0, sl_), right = prmt(loaded, own X1, sr_)
+    if (redge && g.mode == ISP_REPEAT) { bon = 1; bcol = 0; bdst = 16 + 8 * G * (lane + 1); }
+    // selectors: left word = prmt(loaded, first own word, sl_), right = prmt(loaded, last own word, sr_)
     uint32_t sl_ = 0x3210, sr_ = 0x3210;
     if (cl && lane == 0) sl_ = g.mode == ISP_CLAMP ? 0x5454 : g.mode == ISP_MIRROR ? 0x5476 : 0x3210;
     if (redge) sr_ = g.mode == ISP_CLAMP ? 0x7676 : g.mode == ISP_MIRROR ? 0x5476 : 0x3210;
@@ -346,7 +351,7 @@ __device__ __forceinline__ void har_band_body(const HarBandParams &p, uint32_t r
         for (int j = 0; j < LR; ++j)
             for (int im = 0; im < 2; ++im) {
                 if (cl && lane == 0) sts32(ring + j * HSLOT + im * HIMG + 12, p.cword);
-                if (redge) sts32(ring + j * HSLOT + im * HIMG + 16 + 8 * (lane + 1), p.cword);
+                if (redge) sts32(ring + j * HSLOT + im * HIMG + 16 + 8 * G * (lane + 1), p.cword);
             }
     }
     const int mcol = active ? x : 0;
@@ -359,18 +364,18 @@ __device__ __forceinline__ void har_band_body(const HarBandParams &p, uint32_t r
             const int yy = map_row1<true>(y0 - 1 + j, g.h, g.mode);
             if (yy < 0) {   // Constant: both staged rows are C
                 for (int im = 0; im < 2; ++im) {
-                    sts32(slot + im * HIMG + 16 + loff, p.cword);
-                    sts32(slot + im * HIMG + 20 + loff, p.cword);
+#pragma unroll
+                    for (int q = 0; q < NWD; ++q) sts32(slot + im * HIMG + 16 + loff + 4 * q, p.cword);
                     if (lane == 0) sts32(slot + im * HIMG + 12, p.cword);
-                    if (lane == 31) sts32(slot + im * HIMG + 16 + 2 * HSTRIP, p.cword);
+                    if (lane == 31) sts32(slot + im * HIMG + 16 + 2 * STRIP, p.cword);
                 }
                 return;
             }
             rx = reinterpret_cast<const char *>(p.dx) + (size_t)yy * pitchb;
             ry = reinterpret_cast<const char *>(p.dy) + (size_t)yy * pitchb;
         }
-        cpa_own<2>(slot + 16 + loff, rx + 2 * mcol, active);
-        cpa_own<2>(slot + HIMG + 16 + loff, ry + 2 * mcol, active);
+        cpa_own<NWD>(slot + 16 + loff, rx + 2 * mcol, active);
+        cpa_own<NWD>(slot + HIMG + 16 + loff, ry + 2 * mcol, active);
         cpa4p(slot + 12, rx + 2 * acol, aon);
         cpa4p(slot + HIMG + 12, ry + 2 * acol, aon);
         cpa4p(slot + bdst, rx + 2 * bcol, bon);
@@ -383,7 +388,7 @@ __device__ __forceinline__ void har_band_body(const HarBandParams &p, uint32_t r
         ny += pitchb;
         cpa_commit();
     }
-    HRow hr[3];
+    HRow hr[3][G];
     uint8_t *orow = p.out + (size_t)y0 * g.out_pitch + x;
     const float2 two = f2(2.f, 2.f);
 #pragma unroll 1
@@ -395,24 +400,35 @@ __device__ __forceinline__ void har_band_body(const HarBandParams &p, uint32_t r
                 cpa_wait<HLD - 1>();
                 __syncwarp();
                 const uint32_t sl = ring + (i & (LR - 1)) * HSLOT + loff;
-                uint32_t X[2], Y[2];
-                lds_own<2>(sl + 16, X);
-                lds_own<2>(sl + HIMG + 16, Y);
-                const uint32_t XL = __byte_perm(lds32(sl + 12), X[0], sl_), YL = __byte_perm(lds32(sl + HIMG + 12), Y[0], sl_);
-                const uint32_t XR = __byte_perm(lds32(sl + 24), X[1], sr_), YR = __byte_perm(lds32(sl + HIMG + 24), Y[1], sr_);
-                hr[k] = har_hrow(XL, X[0], X[1], XR, YL, Y[0], Y[1], YR);
+                uint32_t X[NWD + 2], Y[NWD + 2];   // [0] left halo word, [1..NWD] own, [NWD+1] right
+                lds_own<NWD>(sl + 16, *reinterpret_cast<uint32_t(*)[NWD]>(&X[1]));
+                lds_own<NWD>(sl + HIMG + 16, *reinterpret_cast<uint32_t(*)[NWD]>(&Y[1]));
+                X[0] = __byte_perm(lds32(sl + 12), X[1], sl_);
+                Y[0] = __byte_perm(lds32(sl + HIMG + 12), Y[1], sl_);
+                X[NWD + 1] = __byte_perm(lds32(sl + 16 + 8 * G), X[NWD], sr_);
+                Y[NWD + 1] = __byte_perm(lds32(sl + HIMG + 16 + 8 * G), Y[NWD], sr_);
+#pragma unroll
+                for (int q = 0; q < G; ++q)
+                    hr[k][q] = har_hrow(X[2 * q], X[2 * q + 1], X[2 * q + 2], X[2 * q + 3], Y[2 * q], Y[2 * q + 1],
+                                        Y[2 * q + 2], Y[2 * q + 3]);
                 if (i >= 2) {
                     // output row y0 + i - 2: rows i-2, i-1, i are hr[k+1], hr[k+2], hr[k] (mod 3)
-                    const HRow &a = hr[(k + 1) % 3], &b = hr[(k + 2) % 3], &c = hr[k];
-                    const float2 sxxE = add2(fma2(two, b.xxE, a.xxE), c.xxE), sxxO = add2(fma2(two, b.xxO, a.xxO), c.xxO);
-                    const float2 syyE = add2(fma2(two, b.yyE, a.yyE), c.yyE), syyO = add2(fma2(two, b.yyO, a.yyO), c.yyO);
-                    const float2 sxyE = add2(fma2(two, b.xyE, a.xyE), c.xyE), sxyO = add2(fma2(two, b.xyO, a.xyO), c.xyO);
-                    uint32_t h0, h1, h2, h3;
-                    harris2p(sxxE, syyE, sxyE, p.thr_f, p.thr_err, p.thr, h0, h2);
-                    harris2p(sxxO, syyO, sxyO, p.thr_f, p.thr_err, p.thr, h1, h3);
-                    if (active)   // bytes (h0, h1, h2, h3)
-                        *reinterpret_cast<uint32_t *>(orow) =
-                            __byte_perm(__byte_perm(h0, h1, 0x0040), __byte_perm(h2, h3, 0x0040), 0x5410);
+                    uint32_t o[G];
+#pragma unroll
+                    for (int q = 0; q < G; ++q) {
+                        const HRow &a = hr[(k + 1) % 3][q], &b = hr[(k + 2) % 3][q], &c = hr[k][q];
+                        const float2 sxxE = add2(fma2(two, b.xxE, a.xxE), c.xxE), sxxO = add2(fma2(two, b.xxO, a.xxO), c.xxO);
+                        const float2 syyE = add2(fma2(two, b.yyE, a.yyE), c.yyE), syyO = add2(fma2(two, b.yyO, a.yyO), c.yyO);
+                        const float2 sxyE = add2(fma2(two, b.xyE, a.xyE), c.xyE), sxyO = add2(fma2(two, b.xyO, a.xyO), c.xyO);
+                        uint32_t h0, h1, h2, h3;
+                        harris2p(sxxE, syyE, sxyE, p.thr_f, p.thr_err, p.thr, h0, h2);
+                        harris2p(sxxO, syyO, sxyO, p.thr_f, p.thr_err, p.thr, h1, h3);
+                        o[q] = __byte_perm(__byte_perm(h0, h1, 0x0040), __byte_perm(h2, h3, 0x0040), 0x5410);
+                    }
+                    if (active) {
+                        if constexpr (G == 2) *reinterpret_cast<uint2 *>(orow) = make_uint2(o[0], o[1]);
+                        else *reinterpret_cast<uint32_t *>(orow) = o[0];
+                    }
                     orow += g.out_pitch;
                 }
                 if (i + HLD < nin) issue(i + HLD, ring + ((i + HLD) & (LR - 1)) * HSLOT);
@@ -424,9 +440,10 @@ __device__ __forceinline__ void har_band_body(const HarBandParams &p, uint32_t r
     }
 }
 
-__global__ void __launch_bounds__(NTB, 4) k_har_band(const __grid_constant__ HarBandParams p)
+template <int G>
+__global__ void __launch_bounds__(NTB, G == 1 ? 4 : 3) k_har_band(const __grid_constant__ HarBandParams p)
 {
-    __shared__ __align__(16) uint8_t rings[BW][LR * HSLOT];
+    __shared__ __align__(16) uint8_t rings[BW][LR * HarShape<G>::SLOT];
     asm volatile("griddepcontrol.wait;" ::: "memory");
     asm volatile("griddepcontrol.launch_dependents;");
     const BandGeom &g = p.g;
@@ -438,8 +455,27 @@ __global__ void __launch_bounds__(NTB, 4) k_har_band(const __grid_constant__ Har
     band_rows(band, g.nband, g.h, y0, y1);
     const bool cl = s < g.sx0, cr = s >= g.sx1, cy = band < g.by0 || band >= g.by1;
     const uint32_t ring = su32(rings[warp]);
-    if (cy) har_band_body<true>(p, ring, s * HSTRIP, y0, y1 - y0, lane, cl, cr);
-    else har_band_body<false>(p, ring, s * HSTRIP, y0, y1 - y0, lane, cl, cr);
+    if (cy) har_band_body<G, true>(p, ring, s * HarShape<G>::STRIP, y0, y1 - y0, lane, cl, cr);
+    else har_band_body<G, false>(p, ring, s * HarShape<G>::STRIP, y0, y1 - y0, lane, cl, cr);
+}
+
+// pixel groups of 4 per lane of the Harris band launch: 2 unless ISP_HARRIS_G=1
+int harris_g()
+{
+    const char *e = getenv("ISP_HARRIS_G");
+    return e && atoi(e) == 1 ? 1 : 2;
+}
+const void *har_band_fn(int gq) { return gq == 1 ? (const void *)k_har_band<1> : (const void *)k_har_band<2>; }
+int har_blocks_per_sm(int gq)
+{
+    static int nb[3] = {-1, -1, -1};
+    if (nb[gq] < 0) {
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb[gq], har_band_fn(gq), NTB, 0) != cudaSuccess) {
+            cudaGetLastError();
+            nb[gq] = 0;
+        }
+    }
+    return nb[gq];
 }
 
 
@@ -1022,7 +1058,7 @@ int band_blocks_per_sm(int which)
 {
     static int nb[5] = {-1, -1, -1, -1, -1};
     if (nb[which] < 0) {
-        const void *fn = which == 1   ? (const void *)k_har_band
+        const void *fn = which == 1   ? har_band_fn(harris_g())
                          : which == 3 ? (const void *)k_fused_band
                          : which == 0 ? (const void *)k_sob_band
                                       : lap_band_fn(which);
@@ -1055,7 +1091,10 @@ void ispi_band_shape(int w, int h, int *tw, int *th)
     *th = (h + g.nband - 1) / g.nband;
 }
 
-int ispi_band_blocks_per_sm(int which) { return band_blocks_per_sm(which == 1 ? 1 : which == 2 ? 0 : band_nw()); }
+int ispi_band_blocks_per_sm(int which)
+{
+    return which == 1 ? har_blocks_per_sm(harris_g()) : band_blocks_per_sm(which == 2 ? 0 : band_nw());
+}
 
 cudaError_t ispi_laplace_band(const uint8_t *img, int w, int h, int pitch, int mode, int cval, uint8_t *out,
                               int out_pitch, cudaStream_t st, int bounds[4])
@@ -1070,18 +1109,21 @@ cudaError_t ispi_laplace_band(const uint8_t *img, int w, int h, int pitch, int m
     return launch_band(lap_band_fn(nw), &p, p.g.ngx * p.g.nband, st);
 }
 
-// Harris band kernel: 4-pixel lane granules of int16 (8-byte aligned rows), 4-byte aligned
-// output rows, h >= 8.
+// Harris band kernel: 4 G-pixel lane granules of int16 (8 G-byte aligned rows), 4 G-byte
+// aligned output rows, h >= 8.
 bool ispi_band_harris_ok(const void *dx, const void *dy, int w, int h, int pitch, const void *out, int out_pitch)
 {
     auto al = [](const void *q, long long pb, int a) { return q && ((uintptr_t)q % a) == 0 && (pb % a) == 0; };
-    return al(dx, 2LL * pitch, 8) && al(dy, 2LL * pitch, 8) && al(out, out_pitch, 4) && w % 4 == 0 && w >= 8 && h >= 8;
+    const int gq = harris_g();
+    return al(dx, 2LL * pitch, 8 * gq) && al(dy, 2LL * pitch, 8 * gq) && al(out, out_pitch, 4 * gq) &&
+           w % (4 * gq) == 0 && w >= 8 * gq && h >= 8;
 }
 
 void ispi_band_harris_shape(int w, int h, int *tw, int *th)
 {
-    const BandGeom g = band_geom(w, h, w, w, ISP_CLAMP, 1, HSTRIP, band_blocks_per_sm(1), bands_hint());
-    *tw = HSTRIP;
+    const int gq = harris_g();
+    const BandGeom g = band_geom(w, h, w, w, ISP_CLAMP, 1, 128 * gq, har_blocks_per_sm(gq), bands_hint());
+    *tw = 128 * gq;
     *th = (h + g.nband - 1) / g.nband;
 }
 
@@ -1089,7 +1131,8 @@ cudaError_t ispi_harris_band(const int16_t *dx, const int16_t *dy, int w, int h,
                              long long thr, uint8_t *out, int out_pitch, cudaStream_t st, int bounds[4])
 {
     HarBandParams p{};
-    p.g = band_geom(w, h, pitch, out_pitch, mode, 1, HSTRIP, band_blocks_per_sm(1), bands_hint());
+    const int gq = harris_g();
+    p.g = band_geom(w, h, pitch, out_pitch, mode, 1, 128 * gq, har_blocks_per_sm(gq), bands_hint());
     p.dx = dx;
     p.dy = dy;
     p.out = out;
@@ -1098,7 +1141,7 @@ cudaError_t ispi_harris_band(const int16_t *dx, const int16_t *dy, int w, int h,
     p.thr_f = (float)p.thr;
     p.thr_err = 2.0f * 5.9604645e-08f * std::fabs(p.thr_f) + 1e-30f;   // |(float)thr - thr| + margin
     bounds[0] = p.g.sx0; bounds[1] = std::max(p.g.sx0, p.g.sx1); bounds[2] = p.g.by0; bounds[3] = p.g.by1;
-    return launch_band((const void *)k_har_band, &p, p.g.ngx * p.g.nband, st);
+    return launch_band(har_band_fn(gq), &p, p.g.ngx * p.g.nband, st);
 }
 
 // Fused cfg3 band kernel: 4-pixel lane granules, 4-byte aligned rows in and out (8-byte for

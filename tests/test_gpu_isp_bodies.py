@@ -528,7 +528,7 @@ def test_laplace_harris_tile_kernels(isp, shape):
             rhar = oracle.harris(rdx, rdy, mode, c, thr)
             got = host(isp.isp_harris_u8(ddx, ddy, mode, c, thr, variant="tma"))
             p = isp.isp_last_plan()
-            assert p["choice"] == CODE["tma"] and p["tile_w"] == 128 and p["tile_h"] < 32, p   # band
+            assert p["choice"] == CODE["tma"] and p["tile_w"] in (128, 256) and p["tile_h"] < 32, p   # band
             np.testing.assert_array_equal(got, rhar, err_msg=f"harris {mode} thr={thr}")
         # random int16 derivatives over the whole Sobel range
         rx = synth.random_i16(h, w, 5)
@@ -563,13 +563,16 @@ def test_laplace_band_kernel(isp, shape, nw, monkeypatch):
     np.testing.assert_array_equal(host(isp.isp_laplace5_u8(d, "mirror", 0)), oracle.laplace5_u8(img, "mirror", 0))
 
 
-@pytest.mark.parametrize("shape", [(8, 8), (9, 132), (70, 2064), (33, 4112), (101, 128), (4096 // 8, 4096), (17, 260)])
-def test_harris_band_kernel(isp, shape):
+@pytest.mark.parametrize("groups", [1, 2])
+@pytest.mark.parametrize("shape", [(8, 16), (9, 136), (70, 2064), (33, 4112), (101, 256), (4096 // 8, 4096), (17, 264)])
+def test_harris_band_kernel(isp, shape, groups, monkeypatch):
     """The warp-strip streaming Harris (band_u8.cu): strips of 128 columns (partial last
     strips down to one lane, one strip that is both L and R), bands down to 4 rows, all
     modes, constants at the ends of the Sobel range, thresholds from far below to far
     above the responses, Sobel derivatives of a structured image and random int16 over the
-    whole range -- bit-exact against the oracle's int64 definition."""
+    whole range -- bit-exact against the oracle's int64 definition; 4 (groups 1) and 8
+    (groups 2) pixels per lane."""
+    monkeypatch.setenv("ISP_HARRIS_G", str(groups))
     h, w = shape
     img = synth.structured_u8(h, w, 23)
     for mode in MODES:
@@ -582,7 +585,7 @@ def test_harris_band_kernel(isp, shape):
                 for thr in (0, -(10 ** 9), 10 ** 8, 10 ** 13):
                     got = host(isp.isp_harris_u8(ddx, ddy, mode, c, thr, variant="tma"))
                     p = isp.isp_last_plan()
-                    assert p["choice"] == CODE["tma"] and p["warp_w"] == 128 and p["tile_h"] < 32, p
+                    assert p["choice"] == CODE["tma"] and p["warp_w"] == 128 * groups and p["tile_h"] < 32, p
                     np.testing.assert_array_equal(got, oracle.harris(dx, dy, mode, c, thr),
                                                   err_msg=f"{mode} c={c} thr={thr}")
 
