@@ -761,19 +761,21 @@ struct SobBandParams {
 
 struct SobP { uint32_t sE, sO, dE, dO; };
 
-template <bool CY>
+template <int G, bool CY>
 __device__ __forceinline__ void sob_band_body(const SobBandParams &p, uint32_t ring, int xs0, int y0, int rows,
                                               int lane, bool cl, bool cr)
 {
+    // G groups of 4 pixels per lane: strips of 128 G columns (BandShape<G>)
+    using B = BandShape<G>;
+    constexpr int LPX = B::LPX, STRIP = B::STRIP, SLOT = B::SLOT;
     const BandGeom &g = p.g;
-    constexpr int LPX = 4;
     const int x = xs0 + LPX * lane;
     const bool active = !cr || x < g.w;
     const bool redge = cr && x + LPX == g.w;
     const int nin = rows + 2;   // >= 6
     const uint32_t loff = LPX * lane;
-    int acol = xs0 - 4, bcol = xs0 + FSTRIP;
-    uint32_t aon = lane == 0 && (!cl || g.mode == ISP_REPEAT), bdst = 16 + FSTRIP, bon = !cr && lane == 31;
+    int acol = xs0 - 4, bcol = xs0 + STRIP;
+    uint32_t aon = lane == 0 && (!cl || g.mode == ISP_REPEAT), bdst = 16 + STRIP, bon = !cr && lane == 31;
     if (cl) acol = g.w - 4;
     if (redge && g.mode == ISP_REPEAT) { bon = 1; bcol = 0; bdst = 16 + LPX * (lane + 1); }
     uint32_t sl_ = 0x3210, sr_ = 0x3210;
@@ -781,8 +783,8 @@ __device__ __forceinline__ void sob_band_body(const SobBandParams &p, uint32_t r
     if (redge) sr_ = g.mode == ISP_CLAMP ? 0x7777 : g.mode == ISP_MIRROR ? 0x0067 : 0x3210;
     if (g.mode == ISP_CONSTANT) {
         for (int j = 0; j < LR; ++j) {
-            if (cl && lane == 0) sts32(ring + j * FSLOT + 12, p.cword);
-            if (redge) sts32(ring + j * FSLOT + 16 + LPX * (lane + 1), p.cword);
+            if (cl && lane == 0) sts32(ring + j * SLOT + 12, p.cword);
+            if (redge) sts32(ring + j * SLOT + 16 + LPX * (lane + 1), p.cword);
         }
     }
     const int mcol = active ? x : 0;
@@ -792,25 +794,28 @@ __device__ __forceinline__ void sob_band_body(const SobBandParams &p, uint32_t r
         if constexpr (CY) {
             const int yy = map_row1<true>(y0 - 1 + j, g.h, g.mode);
             if (yy < 0) {
-                sts32(slot + 16 + loff, p.cword);
+#pragma unroll
+                for (int q = 0; q < G; ++q) sts32(slot + 16 + loff + 4 * q, p.cword);
                 if (lane == 0) sts32(slot + 12, p.cword);
-                if (lane == 31) sts32(slot + 16 + FSTRIP, p.cword);
+                if (lane == 31) sts32(slot + 16 + STRIP, p.cword);
                 return;
             }
             rp = p.img + (size_t)yy * g.pitch;
         }
-        cpa4p(slot + 16 + loff, rp + mcol, active);
+        if constexpr (G == 1) cpa4p(slot + 16 + loff, rp + mcol, active);
+        else cpa_own<G>(slot + 16 + loff, rp + mcol, active);
         cpa4p(slot + 12, rp + acol, aon);
         cpa4p(slot + bdst, rp + bcol, bon);
     };
 #pragma unroll
     for (int j = 0; j < FLD; ++j) {
-        issue(j, ring + j * FSLOT);
+        issue(j, ring + j * SLOT);
         nrp += g.pitch;
         cpa_commit();
     }
-    SobP sr[3];
+    SobP sr[3][G];
     ptrdiff_t o2 = (ptrdiff_t)(y0 - 2) * g.out_pitch + x;   // output offset of row y0 + i - 2
+    const float2 M = f2(12582912.f, 12582912.f);
 #pragma unroll 1
     for (int i0 = 0; i0 < nin; i0 += 3) {
 #pragma unroll
@@ -819,46 +824,62 @@ __device__ __forceinline__ void sob_band_body(const SobBandParams &p, uint32_t r
             if (i < nin) {
                 cpa_wait<FLD - 1>();
                 __syncwarp();
-                const uint32_t sl = ring + (i & (LR - 1)) * FSLOT + loff;
-                const uint32_t W0 = lds32(sl + 16);
-                const uint32_t L = __byte_perm(lds32(sl + 12), W0, sl_), R = __byte_perm(lds32(sl + 20), W0, sr_);
-                const uint32_t F0 = __funnelshift_r(L, W0, 16), F1 = __funnelshift_r(W0, R, 16);
-                const uint32_t Om2 = od(F0), E0 = ev(W0), O0 = od(W0), E2 = ev(F1);
-                SobP &sh = sr[k];
-                sh.sE = Om2 + 2u * E0 + O0;
-                sh.sO = E0 + 2u * O0 + E2;
-                sh.dE = O0 + 0x01000100u - Om2;
-                sh.dO = E2 + 0x01000100u - E0;
+                const uint32_t sl = ring + (i & (LR - 1)) * SLOT + loff;
+                uint32_t W[G + 2];   // [0] left halo word, [1..G] own, [G+1] right
+                if constexpr (G == 1) W[1] = lds32(sl + 16);
+                else lds_own<G>(sl + 16, *reinterpret_cast<uint32_t(*)[G]>(&W[1]));
+                W[0] = __byte_perm(lds32(sl + 12), W[1], sl_);
+                W[G + 1] = __byte_perm(lds32(sl + 16 + LPX), W[G], sr_);
+#pragma unroll
+                for (int q = 0; q < G; ++q) {
+                    const uint32_t F0 = __funnelshift_r(W[q], W[q + 1], 16), F1 = __funnelshift_r(W[q + 1], W[q + 2], 16);
+                    const uint32_t Om2 = od(F0), E0 = ev(W[q + 1]), O0 = od(W[q + 1]), E2 = ev(F1);
+                    SobP &sh = sr[k][q];
+                    sh.sE = Om2 + 2u * E0 + O0;
+                    sh.sO = E0 + 2u * O0 + E2;
+                    sh.dE = O0 + 0x01000100u - Om2;
+                    sh.dO = E2 + 0x01000100u - E0;
+                }
                 if (i >= 2) {   // row y0 + i - 2 from rows i-2, i-1, i
-                    const SobP &a = sr[(k + 1) % 3], &b = sr[(k + 2) % 3];
-                    const uint32_t dxE = a.dE + 2u * b.dE + sh.dE, dxO = a.dO + 2u * b.dO + sh.dO;
-                    const uint32_t dyE = sh.sE + 0x04000400u - a.sE, dyO = sh.sO + 0x04000400u - a.sO;
-                    const float2 xE = lanes_f(dxE, 1024.f), xO = lanes_f(dxO, 1024.f);
-                    const float2 yE = lanes_f(dyE, 1024.f), yO = lanes_f(dyO, 1024.f);
-                    if (p.mag) {
-                        const float2 nE = fma2(xE, xE, mul2(yE, yE)), nO = fma2(xO, xO, mul2(yO, yO));
-                        const uint32_t m0 = mag_bits(nE.x), m1 = mag_bits(nO.x), m2 = mag_bits(nE.y), m3 = mag_bits(nO.y);
-                        const uint32_t mw =
-                            __byte_perm(__byte_perm(m0, m1, 0x0040), __byte_perm(m2, m3, 0x0040), 0x5410);
-                        if (active) *reinterpret_cast<uint32_t *>(p.mag + o2) = mw;
+                    uint32_t mw[G], dxw[2 * G], dyw[2 * G];
+#pragma unroll
+                    for (int q = 0; q < G; ++q) {
+                        const SobP &a = sr[(k + 1) % 3][q], &b = sr[(k + 2) % 3][q], &sh = sr[k][q];
+                        const uint32_t dxE = a.dE + 2u * b.dE + sh.dE, dxO = a.dO + 2u * b.dO + sh.dO;
+                        const uint32_t dyE = sh.sE + 0x04000400u - a.sE, dyO = sh.sO + 0x04000400u - a.sO;
+                        const float2 xE = lanes_f(dxE, 1024.f), xO = lanes_f(dxO, 1024.f);
+                        const float2 yE = lanes_f(dyE, 1024.f), yO = lanes_f(dyO, 1024.f);
+                        if (p.mag) {
+                            const float2 nE = fma2(xE, xE, mul2(yE, yE)), nO = fma2(xO, xO, mul2(yO, yO));
+                            const uint32_t m0 = mag_bits(nE.x), m1 = mag_bits(nO.x), m2 = mag_bits(nE.y),
+                                           m3 = mag_bits(nO.y);
+                            mw[q] = __byte_perm(__byte_perm(m0, m1, 0x0040), __byte_perm(m2, m3, 0x0040), 0x5410);
+                        }
+                        if (p.dx) {   // int16 = low half of the bits of v + 1.5 * 2^23
+                            const float2 a2 = add2(xE, M), b2 = add2(xO, M);
+                            dxw[2 * q] = __byte_perm(__float_as_uint(a2.x), __float_as_uint(b2.x), 0x5410);
+                            dxw[2 * q + 1] = __byte_perm(__float_as_uint(a2.y), __float_as_uint(b2.y), 0x5410);
+                        }
+                        if (p.dy) {
+                            const float2 a2 = add2(yE, M), b2 = add2(yO, M);
+                            dyw[2 * q] = __byte_perm(__float_as_uint(a2.x), __float_as_uint(b2.x), 0x5410);
+                            dyw[2 * q + 1] = __byte_perm(__float_as_uint(a2.y), __float_as_uint(b2.y), 0x5410);
+                        }
                     }
-                    if (p.dx) {   // int16 = low half of the bits of v + 1.5 * 2^23
-                        const float2 a2 = add2(xE, f2(12582912.f, 12582912.f)), b2 = add2(xO, f2(12582912.f, 12582912.f));
-                        if (active)
-                            *reinterpret_cast<uint2 *>(p.dx + o2) =
-                                make_uint2(__byte_perm(__float_as_uint(a2.x), __float_as_uint(b2.x), 0x5410),
-                                           __byte_perm(__float_as_uint(a2.y), __float_as_uint(b2.y), 0x5410));
-                    }
-                    if (p.dy) {
-                        const float2 a2 = add2(yE, f2(12582912.f, 12582912.f)), b2 = add2(yO, f2(12582912.f, 12582912.f));
-                        if (active)
-                            *reinterpret_cast<uint2 *>(p.dy + o2) =
-                                make_uint2(__byte_perm(__float_as_uint(a2.x), __float_as_uint(b2.x), 0x5410),
-                                           __byte_perm(__float_as_uint(a2.y), __float_as_uint(b2.y), 0x5410));
+                    if (active) {
+                        if constexpr (G == 2) {
+                            if (p.mag) *reinterpret_cast<uint2 *>(p.mag + o2) = make_uint2(mw[0], mw[1]);
+                            if (p.dx) *reinterpret_cast<uint4 *>(p.dx + o2) = make_uint4(dxw[0], dxw[1], dxw[2], dxw[3]);
+                            if (p.dy) *reinterpret_cast<uint4 *>(p.dy + o2) = make_uint4(dyw[0], dyw[1], dyw[2], dyw[3]);
+                        } else {
+                            if (p.mag) *reinterpret_cast<uint32_t *>(p.mag + o2) = mw[0];
+                            if (p.dx) *reinterpret_cast<uint2 *>(p.dx + o2) = make_uint2(dxw[0], dxw[1]);
+                            if (p.dy) *reinterpret_cast<uint2 *>(p.dy + o2) = make_uint2(dyw[0], dyw[1]);
+                        }
                     }
                 }
                 o2 += g.out_pitch;
-                if (i + FLD < nin) issue(i + FLD, ring + ((i + FLD) & (LR - 1)) * FSLOT);
+                if (i + FLD < nin) issue(i + FLD, ring + ((i + FLD) & (LR - 1)) * SLOT);
                 nrp += g.pitch;
                 cpa_commit();
             }
@@ -866,9 +887,10 @@ __device__ __forceinline__ void sob_band_body(const SobBandParams &p, uint32_t r
     }
 }
 
+template <int G>
 __global__ void __launch_bounds__(NTB, 8) k_sob_band(const __grid_constant__ SobBandParams p)
 {
-    __shared__ __align__(16) uint8_t rings[BW][LR * FSLOT];
+    __shared__ __align__(16) uint8_t rings[BW][LR * BandShape<G>::SLOT];
     asm volatile("griddepcontrol.wait;" ::: "memory");
     asm volatile("griddepcontrol.launch_dependents;");
     const BandGeom &g = p.g;
@@ -880,10 +902,28 @@ __global__ void __launch_bounds__(NTB, 8) k_sob_band(const __grid_constant__ Sob
     band_rows(band, g.nband, g.h, y0, y1);
     const bool cl = s < g.sx0, cr = s >= g.sx1, cy = band < g.by0 || band >= g.by1;
     const uint32_t ring = su32(rings[warp]);
-    if (cy) sob_band_body<true>(p, ring, s * FSTRIP, y0, y1 - y0, lane, cl, cr);
-    else sob_band_body<false>(p, ring, s * FSTRIP, y0, y1 - y0, lane, cl, cr);
+    if (cy) sob_band_body<G, true>(p, ring, s * BandShape<G>::STRIP, y0, y1 - y0, lane, cl, cr);
+    else sob_band_body<G, false>(p, ring, s * BandShape<G>::STRIP, y0, y1 - y0, lane, cl, cr);
 }
 
+// pixel groups of 4 per lane of the Sobel band launch: 2 unless ISP_SOBEL_G=1
+int sobel_g()
+{
+    const char *e = getenv("ISP_SOBEL_G");
+    return e && atoi(e) == 1 ? 1 : 2;
+}
+const void *sob_band_fn(int gq) { return gq == 1 ? (const void *)k_sob_band<1> : (const void *)k_sob_band<2>; }
+int sob_blocks_per_sm(int gq)
+{
+    static int nb[3] = {-1, -1, -1};
+    if (nb[gq] < 0) {
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb[gq], sob_band_fn(gq), NTB, 0) != cudaSuccess) {
+            cudaGetLastError();
+            nb[gq] = 0;
+        }
+    }
+    return nb[gq];
+}
 
 // ------------------------------------------------------------------------------ separable u8
 // Separable u8 masks with non-negative integer weights whose products sum to at most the
@@ -1060,7 +1100,7 @@ int band_blocks_per_sm(int which)
     if (nb[which] < 0) {
         const void *fn = which == 1   ? har_band_fn(harris_g())
                          : which == 3 ? (const void *)k_fused_band
-                         : which == 0 ? (const void *)k_sob_band
+                         : which == 0 ? sob_band_fn(sobel_g())
                                       : lap_band_fn(which);
         if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb[which], fn, NTB, 0) != cudaSuccess) {
             cudaGetLastError();
@@ -1093,7 +1133,8 @@ void ispi_band_shape(int w, int h, int *tw, int *th)
 
 int ispi_band_blocks_per_sm(int which)
 {
-    return which == 1 ? har_blocks_per_sm(harris_g()) : band_blocks_per_sm(which == 2 ? 0 : band_nw());
+    return which == 1 ? har_blocks_per_sm(harris_g()) : which == 2 ? sob_blocks_per_sm(sobel_g())
+                                                              : band_blocks_per_sm(band_nw());
 }
 
 cudaError_t ispi_laplace_band(const uint8_t *img, int w, int h, int pitch, int mode, int cval, uint8_t *out,
@@ -1172,20 +1213,22 @@ cudaError_t ispi_fused_band(const uint8_t *img, int w, int h, int pitch, int mod
     return launch_band((const void *)k_fused_band, &p, p.g.ngx * p.g.nband, st);
 }
 
-// Sobel band kernel: 4-pixel lane granules, 4-byte aligned input rows, 4-byte aligned mag
-// rows and 8-byte aligned dx / dy rows, h >= 8.
+// Sobel band kernel: 4 G-pixel lane granules, 4 G-byte aligned input and mag rows, 8 G-byte
+// aligned dx / dy rows, h >= 8.
 bool ispi_band_sobel_ok(const void *img, int w, int h, int pitch, const void *dx, const void *dy, const void *mag,
                         int out_pitch)
 {
     auto al = [](const void *q, long long pb, int a) { return ((uintptr_t)q % a) == 0 && (pb % a) == 0; };
-    return al(img, pitch, 4) && (!mag || al(mag, out_pitch, 4)) && (!dx || al(dx, 2LL * out_pitch, 8)) &&
-           (!dy || al(dy, 2LL * out_pitch, 8)) && w % 4 == 0 && w >= 8 && h >= 8;
+    const int gq = sobel_g(), v = 4 * gq;
+    return al(img, pitch, v) && (!mag || al(mag, out_pitch, v)) && (!dx || al(dx, 2LL * out_pitch, 2 * v)) &&
+           (!dy || al(dy, 2LL * out_pitch, 2 * v)) && w % v == 0 && w >= 2 * v && h >= 8;
 }
 
 void ispi_band_sobel_shape(int w, int h, int *tw, int *th)
 {
-    const BandGeom g = band_geom(w, h, w, w, ISP_CLAMP, 1, FSTRIP, band_blocks_per_sm(0), bands_hint());
-    *tw = FSTRIP;
+    const int gq = sobel_g();
+    const BandGeom g = band_geom(w, h, w, w, ISP_CLAMP, 1, 128 * gq, sob_blocks_per_sm(gq), bands_hint());
+    *tw = 128 * gq;
     *th = (h + g.nband - 1) / g.nband;
 }
 
@@ -1193,12 +1236,13 @@ cudaError_t ispi_sobel_band(const uint8_t *img, int w, int h, int pitch, int mod
                             uint8_t *mag, int out_pitch, cudaStream_t st, int bounds[4])
 {
     SobBandParams p{};
-    p.g = band_geom(w, h, pitch, out_pitch, mode, 1, FSTRIP, band_blocks_per_sm(0), bands_hint());
+    const int gq = sobel_g();
+    p.g = band_geom(w, h, pitch, out_pitch, mode, 1, 128 * gq, sob_blocks_per_sm(gq), bands_hint());
     p.img = img;
     p.dx = dx; p.dy = dy; p.mag = mag;
     p.cword = 0x01010101u * (uint32_t)(cval & 0xff);
     bounds[0] = p.g.sx0; bounds[1] = std::max(p.g.sx0, p.g.sx1); bounds[2] = p.g.by0; bounds[3] = p.g.by1;
-    return launch_band((const void *)k_sob_band, &p, p.g.ngx * p.g.nband, st);
+    return launch_band(sob_band_fn(gq), &p, p.g.ngx * p.g.nband, st);
 }
 
 // Separable u8 band kernel eligibility: K = 3 / 5, non-negative weights, divisor 2^s <= 256

@@ -615,12 +615,14 @@ def test_sep_band_kernel(isp, shape, m):
 
 
 # ---------------------------------------------------------------- warp-strip band Sobel
-@pytest.mark.parametrize("shape", [(8, 8), (9, 132), (70, 2064), (45, 260), (4096 // 8, 4096)])
-def test_sobel_band_kernel(isp, shape):
+@pytest.mark.parametrize("groups", [1, 2])
+@pytest.mark.parametrize("shape", [(8, 16), (9, 136), (70, 2064), (45, 264), (4096 // 8, 4096)])
+def test_sobel_band_kernel(isp, shape, groups, monkeypatch):
     """k_sob_band (band_u8.cu), the TMA / AUTO kernel of isp_sobel_u8: strips of 128
     columns (partial last strips down to one lane, one strip that is L and R), all modes and
     constants 0 / 255, every subset of the dx / dy / mag outputs -- bit-exact against the
-    oracle, the plan showing the band kernel."""
+    oracle, the plan showing the band kernel; 4 (groups 1) and 8 (groups 2) pixels per lane."""
+    monkeypatch.setenv("ISP_SOBEL_G", str(groups))
     h, w = shape
     img = synth.structured_u8(h, w, 41)
     img[0, :] = 255
@@ -632,7 +634,7 @@ def test_sobel_band_kernel(isp, shape):
             for want in (("dx", "dy", "mag"), ("mag",), ("dx",), ("dy", "mag")):
                 dx, dy, mag = isp.isp_sobel_u8(d, mode, c, variant="tma", want=want)
                 p = isp.isp_last_plan()
-                assert p["choice"] == CODE["tma"] and p["warp_w"] == 128 and p["tile_h"] < 32, p
+                assert p["choice"] == CODE["tma"] and p["warp_w"] == 128 * groups and p["tile_h"] < 32, p
                 for name, got, ref in (("dx", dx, rdx), ("dy", dy, rdy), ("mag", mag, rmag)):
                     if name in want:
                         np.testing.assert_array_equal(host(got), ref, err_msg=f"{name} {mode} c={c} {want}")
