@@ -944,11 +944,10 @@ struct SepU8BandParams {
     int shift;           // s: d = 2^s
 };
 
-template <int K, bool CY>
+template <int NW, int K, bool CY>
 __device__ __forceinline__ void sepu8_band_body(const SepU8BandParams &p, uint32_t ring, int xs0, int y0, int rows,
                                                 int lane, bool cl, bool cr)
 {
-    constexpr int NW = 2;
     using B = BandShape<NW>;
     constexpr int LPX = B::LPX, STRIP = B::STRIP, SLOT = B::SLOT, HY = K / 2;
     const BandGeom &g = p.g;
@@ -1011,24 +1010,26 @@ __device__ __forceinline__ void sepu8_band_body(const SepU8BandParams &p, uint32
                 lds_own<NW>(sl + 16, *reinterpret_cast<uint32_t(*)[NW]>(&W[1]));
                 W[0] = __byte_perm(lds32(sl + 12), W[1], sl_);
                 W[NW + 1] = __byte_perm(lds32(sl + 16 + LPX), W[NW], sr_);
-                // byte windows F[j] = bytes j-2 .. j+1 relative to the lane's pixel 0, j = 0..8
-                uint32_t F[9];
+                // byte windows F[j] = bytes j-2 .. j+1 relative to the lane's pixel 0, j = 0..4 NW
+                constexpr int NPX = 4 * NW;
+                uint32_t F[NPX + 1];
 #pragma unroll
-                for (int j = 0; j < 9; ++j) {
+                for (int j = 0; j <= NPX; ++j) {
                     const int q = (j + 2) >> 2, sh = (j + 2) & 3;   // window starts in word q-1 ... of W (offset -4)
                     F[j] = sh == 0 ? W[q] : __funnelshift_r(W[q], W[q + 1], 8 * sh);
                 }
-                uint32_t H[8];
+                uint32_t H[NPX];
 #pragma unroll
-                for (int px = 0; px < 8; ++px) {
+                for (int px = 0; px < NPX; ++px) {
                     if constexpr (K == 5) H[px] = __dp4a(F[px + 1], p.r4w, __dp4a(F[px], p.r03, 0u));   // bytes px-2..px+2
                     else H[px] = __dp4a(F[px + 1], p.r03, 0u);                                        // bytes px-1..px+1
                 }
                 uint32_t(&hn)[2 * NW] = hr[k];
-                hn[0] = H[2] * 65536u + H[0];
-                hn[1] = H[3] * 65536u + H[1];
-                hn[2] = H[6] * 65536u + H[4];
-                hn[3] = H[7] * 65536u + H[5];
+#pragma unroll
+                for (int q = 0; q < NW; ++q) {
+                    hn[2 * q] = H[4 * q + 2] * 65536u + H[4 * q];
+                    hn[2 * q + 1] = H[4 * q + 3] * 65536u + H[4 * q + 1];
+                }
                 if (i >= K - 1 && active) {
                     // output row y0 + i - (K-1): rows i-K+1 .. i = ring slots (k+1+j) % K
                     uint32_t v[2 * NW];
@@ -1039,7 +1040,13 @@ __device__ __forceinline__ void sepu8_band_body(const SepU8BandParams &p, uint32
                         for (int j = 0; j < K; ++j) a += (uint32_t)p.col[j] * hr[(k + 1 + j) % K][q];
                         v[q] = (a >> p.shift) & 0x00FF00FFu;
                     }
-                    *reinterpret_cast<uint2 *>(orow) = make_uint2(__byte_perm(v[0], v[1], 0x6240), __byte_perm(v[2], v[3], 0x6240));
+                    if constexpr (NW == 4)
+                        *reinterpret_cast<uint4 *>(orow) =
+                            make_uint4(__byte_perm(v[0], v[1], 0x6240), __byte_perm(v[2], v[3], 0x6240),
+                                       __byte_perm(v[4], v[5], 0x6240), __byte_perm(v[6], v[7], 0x6240));
+                    else
+                        *reinterpret_cast<uint2 *>(orow) =
+                            make_uint2(__byte_perm(v[0], v[1], 0x6240), __byte_perm(v[2], v[3], 0x6240));
                 }
                 orow += g.out_pitch;
                 if (i + LD < nin) issue(i + LD, ring + ((i + LD) & (LR - 1)) * SLOT);
@@ -1050,10 +1057,10 @@ __device__ __forceinline__ void sepu8_band_body(const SepU8BandParams &p, uint32
     }
 }
 
-template <int K>
-__global__ void __launch_bounds__(NTB, 8) k_sepu8_band(const __grid_constant__ SepU8BandParams p)
+template <int NW, int K>
+__global__ void __launch_bounds__(NTB, NW == 2 ? 8 : 5) k_sepu8_band(const __grid_constant__ SepU8BandParams p)
 {
-    __shared__ __align__(16) uint8_t rings[BW][LR * BandShape<2>::SLOT];
+    __shared__ __align__(16) uint8_t rings[BW][LR * BandShape<NW>::SLOT];
     asm volatile("griddepcontrol.wait;" ::: "memory");
     asm volatile("griddepcontrol.launch_dependents;");
     const BandGeom &g = p.g;
@@ -1065,16 +1072,29 @@ __global__ void __launch_bounds__(NTB, 8) k_sepu8_band(const __grid_constant__ S
     band_rows(band, g.nband, g.h, y0, y1);
     const bool cl = s < g.sx0, cr = s >= g.sx1, cy = band < g.by0 || band >= g.by1;
     const uint32_t ring = su32(rings[warp]);
-    if (cy) sepu8_band_body<K, true>(p, ring, s * BandShape<2>::STRIP, y0, y1 - y0, lane, cl, cr);
-    else sepu8_band_body<K, false>(p, ring, s * BandShape<2>::STRIP, y0, y1 - y0, lane, cl, cr);
+    if (cy) sepu8_band_body<NW, K, true>(p, ring, s * BandShape<NW>::STRIP, y0, y1 - y0, lane, cl, cr);
+    else sepu8_band_body<NW, K, false>(p, ring, s * BandShape<NW>::STRIP, y0, y1 - y0, lane, cl, cr);
+}
+
+// words (4 pixels) per lane of the separable u8 band launch: 4 unless ISP_SEPU8_NW=2
+int sepu8_nw()
+{
+    const char *e = getenv("ISP_SEPU8_NW");
+    return e && atoi(e) == 2 ? 2 : 4;
+}
+const void *sepu8_fn(int nw, int k)
+{
+    if (nw == 2) return k == 5 ? (const void *)k_sepu8_band<2, 5> : (const void *)k_sepu8_band<2, 3>;
+    return k == 5 ? (const void *)k_sepu8_band<4, 5> : (const void *)k_sepu8_band<4, 3>;
 }
 
 int sepu8_blocks_per_sm(int k)
 {
-    static int nb[2] = {-1, -1};
-    int &v = nb[k == 5];
+    static int nb[2][2] = {{-1, -1}, {-1, -1}};
+    const int nw = sepu8_nw();
+    int &v = nb[nw == 4][k == 5];
     if (v < 0) {
-        const void *fn = k == 5 ? (const void *)k_sepu8_band<5> : (const void *)k_sepu8_band<3>;
+        const void *fn = sepu8_fn(nw, k);
         if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&v, fn, NTB, 0) != cudaSuccess) {
             cudaGetLastError();
             v = 0;
@@ -1259,13 +1279,15 @@ bool ispi_sepu8_band_ok(const void *img, int w, int h, int pitch, const void *ou
         sr += row[i];
         sc += col[i];
     }
-    return sr * sc <= divisor && al(img, pitch, 8) && al(out, out_pitch, 8) && w % 8 == 0 && w >= 16 && h >= 8;
+    const int v = 4 * sepu8_nw();
+    return sr * sc <= divisor && al(img, pitch, v) && al(out, out_pitch, v) && w % v == 0 && w >= 2 * v && h >= 8;
 }
 
 void ispi_sepu8_band_shape(int w, int h, int k, int *tw, int *th)
 {
-    const BandGeom g = band_geom(w, h, w, w, ISP_CLAMP, k / 2, 256, sepu8_blocks_per_sm(k), bands_hint());
-    *tw = 256;
+    const int strip = 128 * sepu8_nw();
+    const BandGeom g = band_geom(w, h, w, w, ISP_CLAMP, k / 2, strip, sepu8_blocks_per_sm(k), bands_hint());
+    *tw = strip;
     *th = (h + g.nband - 1) / g.nband;
 }
 
@@ -1275,7 +1297,8 @@ cudaError_t ispi_sepu8_band(const uint8_t *img, int w, int h, int pitch, int k, 
                             int divisor, int mode, int cval, uint8_t *out, int out_pitch, cudaStream_t st, int bounds[4])
 {
     SepU8BandParams p{};
-    p.g = band_geom(w, h, pitch, out_pitch, mode, k / 2, 256, sepu8_blocks_per_sm(k), bands_hint());
+    const int nw = sepu8_nw();
+    p.g = band_geom(w, h, pitch, out_pitch, mode, k / 2, 128 * nw, sepu8_blocks_per_sm(k), bands_hint());
     p.img = img;
     p.out = out;
     p.cword = 0x01010101u * (uint32_t)(cval & 0xff);
@@ -1291,5 +1314,5 @@ cudaError_t ispi_sepu8_band(const uint8_t *img, int w, int h, int pitch, int k, 
     while ((1 << s) < divisor) ++s;
     p.shift = s;
     bounds[0] = p.g.sx0; bounds[1] = std::max(p.g.sx0, p.g.sx1); bounds[2] = p.g.by0; bounds[3] = p.g.by1;
-    return launch_band(k == 5 ? (const void *)k_sepu8_band<5> : (const void *)k_sepu8_band<3>, &p, p.g.ngx * p.g.nband, st);
+    return launch_band(sepu8_fn(nw, k), &p, p.g.ngx * p.g.nband, st);
 }

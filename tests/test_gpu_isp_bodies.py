@@ -641,12 +641,15 @@ def test_sobel_band_kernel(isp, shape, groups, monkeypatch):
 
 
 # ---------------------------------------------------------------- warp-strip band separable u8
-@pytest.mark.parametrize("shape", [(8, 16), (9, 48), (70, 2064), (33, 4112), (260, 528), (4096 // 8, 4096)])
-def test_sepu8_band_kernel(isp, shape):
+@pytest.mark.parametrize("nw", [2, 4])
+@pytest.mark.parametrize("shape", [(8, 32), (9, 48), (70, 2064), (33, 4112), (260, 528), (4096 // 8, 4096)])
+def test_sepu8_band_kernel(isp, shape, nw, monkeypatch):
     """k_sepu8_band (band_u8.cu), the TMA / AUTO kernel of normalised separable u8 masks: the
     3x3 / 16 and 5x5 / 256 binomials and a [1,2,1]^2 / 32 mask (result <= 127), all modes,
     strips of 256 columns with partial last strips -- bit-exact against the oracle, the plan
-    showing the band kernel; a divisor that is not a power of two takes the generic path."""
+    showing the band kernel; a divisor that is not a power of two takes the generic path;
+    8 (nw 2) and 16 (nw 4) pixels per lane."""
+    monkeypatch.setenv("ISP_SEPU8_NW", str(nw))
     h, w = shape
     img = synth.uniform_u8(h, w, 51)
     img[0, :] = 255
@@ -658,9 +661,9 @@ def test_sepu8_band_kernel(isp, shape):
             ref = oracle.filter_u8(img, mask, div, mode, 201)
             got = host(isp.isp_filter_u8(d, mask, div, mode, 201, variant="tma"))
             p = isp.isp_last_plan()
-            assert p["choice"] == CODE["tma"] and p["warp_w"] == 256 and p["tile_h"] < 32, p
+            assert p["choice"] == CODE["tma"] and p["warp_w"] == 128 * nw and p["tile_h"] < 32, p
             np.testing.assert_array_equal(got, ref, err_msg=f"{mode} div={div} m={mask.shape}")
     mask, _ = oracle.gaussian_u8_mask(5)
     got = host(isp.isp_filter_u8(d, mask, 300, "mirror", 0, variant="tma"))
-    assert isp.isp_last_plan()["warp_w"] != 256
+    assert isp.isp_last_plan()["warp_w"] != 128 * nw
     np.testing.assert_array_equal(got, oracle.filter_u8(img, mask, 300, "mirror", 0))

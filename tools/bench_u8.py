@@ -16,6 +16,9 @@ import torch  # noqa: E402
 
 import paper_conf_ipps_qiaoth21_b200 as isp  # noqa: E402
 import synth  # noqa: E402
+import numpy as np  # noqa: E402
+
+G5 = np.outer(synth.binomial_row(5), synth.binomial_row(5)).astype(np.int32)
 
 
 def timed(fn, R=12, reps=20):
@@ -73,6 +76,7 @@ def main():
                 ("sobel", 6, lambda i: isp.isp_sobel_u8(imgs[i % nb], a.mode, dx=dxs[i % nb], dy=dys[i % nb],
                                                         mag=o1[i % nb], variant=v)),
                 ("copy", 2, lambda i: o2[i % nb].copy_(imgs[i % nb])),   # torch copy of the same bytes
+                ("gauss5", 2, lambda i: isp.isp_filter_u8(imgs[i % nb], G5, 256, a.mode, out=o2[i % nb], variant=v)),
                 ("laplace", 2, lambda i: isp.isp_laplace5_u8(imgs[i % nb], a.mode, out=o2[i % nb], variant=v)),
                 ("harris", 5, lambda i: isp.isp_harris_u8(dxs[i % nb], dys[i % nb], a.mode, out=o3[i % nb], variant=v)),
             ]:
