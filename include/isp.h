@@ -47,10 +47,14 @@ typedef enum { ISP_U8 = 0, ISP_I16 = 1, ISP_I32 = 2, ISP_F32 = 3 } isp_dtype_t;
 /* ISP_AUTO = "isp+m": the model of Eq. (10) picks ISP or NAIVE; its ISP is
  * ISP_TMA where eligible, else ISP_WARP.  ISP_BLOCK = Listing 3 and ISP_WARP = Listing 5
  * on the register-streaming kernels (per-read checks only where a region needs them);
- * ISP_TMA = Listing 3 on the TMA-staged kernels (bulk async copies into shared memory;
- * checks only in the staging of border blocks, reading A21; needs 16-B aligned rows and
- * a compiled window, else runs as ISP_BLOCK); ISP_NAIVE = all four checks on every read
- * (Eq. 3 baseline). */
+ * ISP_TMA = Listing 3 on the staged kernels: for separable f32 masks (images and strips),
+ * normalised separable u8 masks, Sobel, Laplace, Harris and the cfg3 pipeline the
+ * warp-strip band kernels (per-warp shared-memory row rings filled by cp.async; a warp's
+ * region from its strip / band: T / B rows mapped once per staged row, L / R edge lanes'
+ * halo words, Body none; A34), otherwise the TMA-staged kernels (bulk async copies into
+ * shared memory; checks only in the staging of border blocks, A21) -- each needs its
+ * alignment (16 B for f32, 4-16 B per lane for u8 / i16) and a compiled window, else runs
+ * as ISP_BLOCK; ISP_NAIVE = all four checks on every read (Eq. 3 baseline). */
 /* Ablations: ISP_SPLIT = one kernel per region (the nine regions launched
  * separately over their block rectangles, instead of the paper's single fat kernel with
  * the Listing-3 switch; plans like ISP_BLOCK); ISP_TEX = texture hardware border
