@@ -614,7 +614,7 @@ __device__ __forceinline__ void fused_band_body(const FusedBandParams &p, uint32
     // by step (pairs (H0,H2), (H1,H3)), bias 6400 per lane carried by the Q ring
     uint32_t lq[3][2] = {}, hp0 = 0, hp1 = 0;
     SobH sr[3];                              // Sobel horizontal parts, ring by step
-    HRow hr[3];                              // Harris horizontal sums of dx / dy row (step - 2)
+    HRow hp, acc;                            // Harris: H(step-1) and H(step-2) + 2 H(step-1)
     const HRow hconst = {f2(p.c4, p.c4), f2(p.c4, p.c4), f2(p.c4, p.c4), f2(p.c4, p.c4), f2(p.c4, p.c4),
                          f2(p.c4, p.c4)};
     const float2 two = f2(2.f, 2.f);
@@ -676,13 +676,13 @@ __device__ __forceinline__ void fused_band_body(const FusedBandParams &p, uint32
                     const float2 yE = lanes_f(dyE, 1024.f), yO = lanes_f(dyO, 1024.f);
                     const float2 xA = lanes_f(xa, 1024.f), xB = lanes_f(xb, 1024.f);
                     const float2 yA = lanes_f(ya, 1024.f), yB = lanes_f(yb, 1024.f);
-                    hr[k] = har_hrow_f(xA, xE, xO, xB, yA, yE, yO, yB);
+                    HRow hn = har_hrow_f(xA, xE, xO, xB, yA, yE, yO, yB);
                     // ... and at remapped rows (the band's first / last dx / dy row)
                     if (i == fix_t) {
-                        if (rep == 2) hr[k] = hconst;
-                        else hr[(k + 2) % 3] = hr[k];   // step 3: row 0 also stands for row -1
+                        if (rep == 2) hn = hconst;
+                        else hp = hn;   // step 3: row 0 also stands for row -1
                     }
-                    if (i == fix_b) hr[k] = rep == 2 ? hconst : hr[(k + 2) % 3];
+                    if (i == fix_b) hn = rep == 2 ? hconst : hp;
                     // ---- magnitude (a9) and the optional dx / dy images of row y0 + i - 3
                     if (i >= 3 && i <= rows + 2) {
                         const ptrdiff_t o3 = o4 + g.out_pitch;
@@ -703,10 +703,10 @@ __device__ __forceinline__ void fused_band_body(const FusedBandParams &p, uint32
                     }
                     if (i >= 4) {
                         // ---- Harris (a10) of row y0 + i - 4: dx / dy rows i-4 .. i-2 (steps)
-                        const HRow &ha = hr[(k + 1) % 3], &hb = hr[(k + 2) % 3], &hc = hr[k];
-                        const float2 sxxE = add2(fma2(two, hb.xxE, ha.xxE), hc.xxE), sxxO = add2(fma2(two, hb.xxO, ha.xxO), hc.xxO);
-                        const float2 syyE = add2(fma2(two, hb.yyE, ha.yyE), hc.yyE), syyO = add2(fma2(two, hb.yyO, ha.yyO), hc.yyO);
-                        const float2 sxyE = add2(fma2(two, hb.xyE, ha.xyE), hc.xyE), sxyO = add2(fma2(two, hb.xyO, ha.xyO), hc.xyO);
+                        // rows i-4 .. i-2 of dx / dy: acc (rows i-4, i-3) + the new row
+                        const float2 sxxE = add2(acc.xxE, hn.xxE), sxxO = add2(acc.xxO, hn.xxO);
+                        const float2 syyE = add2(acc.yyE, hn.yyE), syyO = add2(acc.yyO, hn.yyO);
+                        const float2 sxyE = add2(acc.xyE, hn.xyE), sxyO = add2(acc.xyO, hn.xyO);
                         uint32_t h0, h1, h2, h3;
                         harris2p(sxxE, syyE, sxyE, p.thr_f, p.thr_err, p.thr, h0, h2);
                         harris2p(sxxO, syyO, sxyO, p.thr_f, p.thr_err, p.thr, h1, h3);
@@ -714,6 +714,14 @@ __device__ __forceinline__ void fused_band_body(const FusedBandParams &p, uint32
                             *reinterpret_cast<uint32_t *>(p.har + o4) =
                                 __byte_perm(__byte_perm(h0, h1, 0x0040), __byte_perm(h2, h3, 0x0040), 0x5410);
                     }
+                    // vertical [1,2,1] as a running pair (two rows of state instead of three;
+                    // integer sums < 2^24, exact in any order)
+                    if (i > 2) {
+                        acc.xxE = fma2(two, hn.xxE, hp.xxE); acc.xxO = fma2(two, hn.xxO, hp.xxO);
+                        acc.yyE = fma2(two, hn.yyE, hp.yyE); acc.yyO = fma2(two, hn.yyO, hp.yyO);
+                        acc.xyE = fma2(two, hn.xyE, hp.xyE); acc.xyO = fma2(two, hn.xyO, hp.xyO);
+                    }
+                    hp = hn;
                 }
                 o4 += g.out_pitch;
                 if (i + FLD < nin) issue(i + FLD, ring + ((i + FLD) & (LR - 1)) * FSLOT);
