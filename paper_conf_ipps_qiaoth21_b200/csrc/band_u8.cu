@@ -512,7 +512,14 @@ struct FusedBandParams {
     float thr_f, thr_err;
 };
 
-constexpr int FSTRIP = 128, FSLOT = 32 + FSTRIP, FLD = 5;
+#ifndef FUSED_FLD
+#define FUSED_FLD 5
+#endif
+#ifndef FUSED_MINB
+#define FUSED_MINB 4
+#endif
+// rows in flight per warp (FLD) and ring slots (FLR >= FLD + 3: rows i-2 .. i+FLD)
+constexpr int FSTRIP = 128, FSLOT = 32 + FSTRIP, FLD = FUSED_FLD, FLR = FLD + 3 <= 8 ? 8 : 16;
 
 struct SobH { uint32_t sA, sE, sO, sB, dA, dE, dO, dB; };
 
@@ -570,7 +577,7 @@ __device__ __forceinline__ void fused_band_body(const FusedBandParams &p, uint32
     if (cl && lane == 0) sl_ = g.mode == ISP_CLAMP ? 0x4444 : g.mode == ISP_MIRROR ? 0x4500 : 0x3210;
     if (redge) sr_ = g.mode == ISP_CLAMP ? 0x7777 : g.mode == ISP_MIRROR ? 0x0067 : 0x3210;
     if (g.mode == ISP_CONSTANT) {
-        for (int j = 0; j < LR; ++j) {
+        for (int j = 0; j < FLR; ++j) {
             if (cl && lane == 0) sts32(ring + j * FSLOT + 12, p.cword);
             if (redge) sts32(ring + j * FSLOT + 16 + LPX * (lane + 1), p.cword);
         }
@@ -627,7 +634,7 @@ __device__ __forceinline__ void fused_band_body(const FusedBandParams &p, uint32
             if (i < nin) {
                 cpa_wait<FLD - 1>();
                 __syncwarp();
-                const uint32_t sl = ring + (i & (LR - 1)) * FSLOT + loff;
+                const uint32_t sl = ring + (i & (FLR - 1)) * FSLOT + loff;
                 const uint32_t W0 = lds32(sl + 16);
                 const uint32_t L = __byte_perm(lds32(sl + 12), W0, sl_), R = __byte_perm(lds32(sl + 20), W0, sr_);
                 const uint32_t F0 = __funnelshift_r(L, W0, 16), F1 = __funnelshift_r(W0, R, 16);
@@ -652,7 +659,7 @@ __device__ __forceinline__ void fused_band_body(const FusedBandParams &p, uint32
                 sh.dO = E2 + 0x01000100u - E0;
                 sh.dB = O2 + 0x01000100u - O0;
                 if (i >= 4) {
-                    const uint32_t c2 = lds32(ring + ((i - 2) & (LR - 1)) * FSLOT + loff + 16);   // row i-2
+                    const uint32_t c2 = lds32(ring + ((i - 2) & (FLR - 1)) * FSLOT + loff + 16);   // row i-2
                     uint32_t vE = box0 - 25u * ev(c2), vO = box1 - 25u * od(c2);
                     asm("max.u16x2 %0, %0, %1;" : "+r"(vE) : "r"(0x19001900u));
                     asm("min.u16x2 %0, %0, %1;" : "+r"(vE) : "r"(0x19FF19FFu));
@@ -724,7 +731,7 @@ __device__ __forceinline__ void fused_band_body(const FusedBandParams &p, uint32
                     hp = hn;
                 }
                 o4 += g.out_pitch;
-                if (i + FLD < nin) issue(i + FLD, ring + ((i + FLD) & (LR - 1)) * FSLOT);
+                if (i + FLD < nin) issue(i + FLD, ring + ((i + FLD) & (FLR - 1)) * FSLOT);
                 nrp += g.pitch;
                 cpa_commit();
             }
@@ -732,9 +739,9 @@ __device__ __forceinline__ void fused_band_body(const FusedBandParams &p, uint32
     }
 }
 
-__global__ void __launch_bounds__(NTB, 4) k_fused_band(const __grid_constant__ FusedBandParams p)
+__global__ void __launch_bounds__(NTB, FUSED_MINB) k_fused_band(const __grid_constant__ FusedBandParams p)
 {
-    __shared__ __align__(16) uint8_t rings[BW][LR * FSLOT];
+    __shared__ __align__(16) uint8_t rings[BW][FLR * FSLOT];
     asm volatile("griddepcontrol.wait;" ::: "memory");
     asm volatile("griddepcontrol.launch_dependents;");
     const BandGeom &g = p.g;
