@@ -315,11 +315,13 @@ __device__ __forceinline__ void harris2p(float2 sxx, float2 syy, float2 sxy, flo
     const float2 t = add2(sxx, syy);
     const float2 tt = mul2(t, t);
     const float2 R = fma2(f2(25.f, 25.f), det, f2(-tt.x, -tt.y));
-    const float2 b = fma2(tt, f2(1.1444091796875e-05f, 1.1444091796875e-05f), f2(thr_err, thr_err));
+    // b = (1 + 2^-10) x the bound, so that |d| >= b decides strictly (and b = 0 only for
+    // t = 0 and thr = 0, where R_f = R25 = 0 is exact: flat areas never take the slow path)
+    const float2 b = fma2(tt, f2(1.14552676677703857421875e-05f, 1.14552676677703857421875e-05f), f2(thr_err, thr_err));
     const float2 d = add2(R, f2(-thr_f, -thr_f));
-    o0 = d.x > b.x ? 255u : 0u;
-    o1 = d.y > b.y ? 255u : 0u;
-    const bool u0 = fabsf(d.x) <= b.x, u1 = fabsf(d.y) <= b.y;   // undecided by the bound
+    o0 = d.x > 0.f ? 255u : 0u;
+    o1 = d.y > 0.f ? 255u : 0u;
+    const bool u0 = fabsf(d.x) < b.x, u1 = fabsf(d.y) < b.y;   // undecided by the bound
     if (__any_sync(0xffffffffu, u0 || u1)) {
         if (u0) o0 = tt.x == 0.f ? (0.0 > thr ? 255u : 0u) : (uint32_t)harris_exact(sxx.x, syy.x, sxy.x, thr);
         if (u1) o1 = tt.y == 0.f ? (0.0 > thr ? 255u : 0u) : (uint32_t)harris_exact(sxx.y, syy.y, sxy.y, thr);
@@ -1215,7 +1217,7 @@ cudaError_t ispi_harris_band(const int16_t *dx, const int16_t *dy, int w, int h,
     p.cword = 0x00010001u * (uint32_t)(uint16_t)(int16_t)cval;
     p.thr = (double)std::max(-9007199254740992ll, std::min(9007199254740992ll, thr));
     p.thr_f = (float)p.thr;
-    p.thr_err = 2.0f * 5.9604645e-08f * std::fabs(p.thr_f) + 1e-30f;   // |(float)thr - thr| + margin
+    p.thr_err = thr_bound(p.thr_f);
     bounds[0] = p.g.sx0; bounds[1] = std::max(p.g.sx0, p.g.sx1); bounds[2] = p.g.by0; bounds[3] = p.g.by1;
     return launch_band(har_band_fn(gq), &p, p.g.ngx * p.g.nband, st);
 }
@@ -1244,7 +1246,7 @@ cudaError_t ispi_fused_band(const uint8_t *img, int w, int h, int pitch, int mod
     p.c4 = 4.0f * (float)hcval * (float)hcval;
     p.thr = (double)std::max(-9007199254740992ll, std::min(9007199254740992ll, thr));
     p.thr_f = (float)p.thr;
-    p.thr_err = 2.0f * 5.9604645e-08f * std::fabs(p.thr_f) + 1e-30f;
+    p.thr_err = thr_bound(p.thr_f);
     return launch_band((const void *)k_fused_band, &p, p.g.ngx * p.g.nband, st);
 }
 

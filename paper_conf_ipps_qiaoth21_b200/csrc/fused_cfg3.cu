@@ -423,11 +423,12 @@ __device__ __forceinline__ void harris2(float2 sxx, float2 syy, float2 sxy, floa
     const float2 tt = mul2(t, t);
     const float2 R = fma2(f2(25.f, 25.f), det, f2(-tt.x, -tt.y));
     const float2 bnd = add2(add2(p, q), tt);
-    const float b0 = fmaf(bnd.x, 7.62939453125e-06f, thr_err), b1 = fmaf(bnd.y, 7.62939453125e-06f, thr_err);
+    // (1 + 2^-10) x the bound: |d| >= b decides strictly (b = 0: flat area, thr = 0, exact)
+    const float b0 = fmaf(bnd.x, 7.6368451118469238281e-06f, thr_err), b1 = fmaf(bnd.y, 7.6368451118469238281e-06f, thr_err);
     const float d0 = R.x - thr_f, d1 = R.y - thr_f;
-    o0 = d0 > b0 ? 255 : 0;
-    o1 = d1 > b1 ? 255 : 0;
-    const bool u0 = fabsf(d0) <= b0, u1 = fabsf(d1) <= b1;     // undecided by the bound
+    o0 = d0 > 0.f ? 255 : 0;
+    o1 = d1 > 0.f ? 255 : 0;
+    const bool u0 = fabsf(d0) < b0, u1 = fabsf(d1) < b1;     // undecided by the bound
     if (__any_sync(0xffffffffu, u0 || u1)) {
         if (u0) o0 = bnd.x == 0.f ? (0.0 > thr ? 255 : 0) : harris_exact(sxx.x, syy.x, sxy.x, thr);
         if (u1) o1 = bnd.y == 0.f ? (0.0 > thr ? 255 : 0) : harris_exact(sxx.y, syy.y, sxy.y, thr);
@@ -595,7 +596,7 @@ __global__ void __launch_bounds__(NT, FUSED_BODY_MINB) k_fused_body(const Params
     const bool full = body || (x + 3 < p.w);
     const double thr = (double)max(-9007199254740992ll, min(9007199254740992ll, p.thr));
     const float thr_f = (float)thr;
-    const float thr_err = 2.0f * 5.9604645e-08f * fabsf(thr_f) + 1e-30f;    // |(float)thr - thr| + margin
+    const float thr_err = 1.1932570487260818e-07f * fabsf(thr_f);   // |(float)thr - thr| x (1 + 2^-10)
     const uint32_t ones = 0x01010101u;
     // Laplace: horizontal 5-sums of staged row sr at the 4 pixels (DP4A on byte windows)
     auto h5 = [&](int sr, int (&H)[4]) {

@@ -32,16 +32,21 @@ __device__ __forceinline__ void harris2(float2 sxx, float2 syy, float2 sxy, floa
     const float2 tt = mul2(t, t);
     const float2 R = fma2(f2(25.f, 25.f), det, f2(-tt.x, -tt.y));
     const float2 bnd = add2(add2(pp, q), tt);
-    const float b0 = fmaf(bnd.x, 7.62939453125e-06f, thr_err), b1 = fmaf(bnd.y, 7.62939453125e-06f, thr_err);
+    // (1 + 2^-10) x the bound: |d| >= b decides strictly; b = 0 only for all-zero sums and
+    // thr = 0, where R_f = R25 = 0 is exact (flat areas never take the slow path)
+    const float b0 = fmaf(bnd.x, 7.6368451118469238281e-06f, thr_err), b1 = fmaf(bnd.y, 7.6368451118469238281e-06f, thr_err);
     const float d0 = R.x - thr_f, d1 = R.y - thr_f;
-    o0 = d0 > b0 ? 255 : 0;
-    o1 = d1 > b1 ? 255 : 0;
-    const bool u0 = fabsf(d0) <= b0, u1 = fabsf(d1) <= b1;
+    o0 = d0 > 0.f ? 255 : 0;
+    o1 = d1 > 0.f ? 255 : 0;
+    const bool u0 = fabsf(d0) < b0, u1 = fabsf(d1) < b1;
     if (__any_sync(0xffffffffu, u0 || u1)) {
         if (u0) o0 = bnd.x == 0.f ? (0.0 > thr ? 255 : 0) : harris_exact(sxx.x, syy.x, sxy.x, thr);
         if (u1) o1 = bnd.y == 0.f ? (0.0 > thr ? 255 : 0) : harris_exact(sxx.y, syy.y, sxy.y, thr);
     }
 }
+
+// |(float)thr - thr| <= 2^-24 |thr| < 2^-23 |thr_f|, inflated by (1 + 2^-10) like the bound
+__host__ __device__ __forceinline__ float thr_bound(float thr_f) { return 1.1932570487260818e-07f * fabsf(thr_f); }
 
 // int16 -> exact float (|v| < 2^22): 1.5 * 2^23 + v has v in its low mantissa bits
 __device__ __forceinline__ float i2f(int v) { return __int_as_float(0x4B400000 + v) - 12582912.0f; }

@@ -220,7 +220,7 @@ __global__ void __launch_bounds__(NT) k_harris_tile(const __grid_constant__ HarP
     if (rbeg >= rend || x >= g.w) return;
     const double thr = (double)max(-9007199254740992ll, min(9007199254740992ll, p.thr));
     const float thr_f = (float)thr;
-    const float thr_err = 2.0f * 5.9604645e-08f * fabsf(thr_f) + 1e-30f;
+    const float thr_err = thr_bound(thr_f);
     HS a = hsum_row(sx, sy, rbeg, xr), b = hsum_row(sx, sy, rbeg + 1, xr);
     const bool full = x + 3 < g.w;
     const float2 two = f2(2.f, 2.f);

@@ -364,6 +364,41 @@ def test_harris_threshold_boundary(isp):
                     np.testing.assert_array_equal(got, ref, err_msg=f"{mode} {v} thr={thr}")
 
 
+def test_harris_flat_areas(isp):
+    """All-zero window sums (flat image areas: t = 0, R25 = 0 exactly) decide in the f32
+    path (the bound is 0 there only for thr = 0): R25 > thr for thr = 0, -1, 1 and far
+    outside, next to textured spots and spots with dy = 0 (R25 = -Sxx^2 < 0), every mode
+    and variant, and the fused pipeline on a piecewise-constant image -- bit-exact."""
+    h, w = 37, 2064
+    dx = np.zeros((h, w), dtype=np.int16)
+    dy = np.zeros((h, w), dtype=np.int16)
+    rng = np.random.default_rng(5)
+    dx[10:14, 300:340] = rng.integers(-1020, 1021, (4, 40))
+    dy[10:14, 300:340] = rng.integers(-1020, 1021, (4, 40))
+    dx[20:23, 1000:1100] = 7          # dy = 0: R25 = -(Sxx)^2
+    dx[0, :] = 1                      # edge row (T region) with tiny sums
+    ddx, ddy = dev(dx), dev(dy)
+    for mode in MODES:
+        for c in ((0, 3) if mode == "constant" else (0,)):
+            for thr in (0, -1, 1, -(10 ** 12), 10 ** 12):
+                ref = oracle.harris(dx, dy, mode, c, thr)
+                for v in ["tma", "warp", "naive"]:
+                    got = host(isp.isp_harris_u8(ddx, ddy, mode, c, thr, variant=v))
+                    ran(isp, v)
+                    np.testing.assert_array_equal(got, ref, err_msg=f"{mode} {v} c={c} thr={thr}")
+    img = np.full((64, 2048), 77, dtype=np.uint8)
+    img[20:30, 500:520] = 200
+    img[40:, :] = 10
+    d = dev(img)
+    for mode in MODES:
+        rdx, rdy, _ = oracle.sobel(img, mode, 0)
+        for thr in (0, -1, 1):
+            want = oracle.harris(rdx, rdy, mode, 0, thr)
+            for v in ["tma", "warp"]:
+                _, _, har = isp.isp_pipeline_cfg3_u8(d, mode, 0, 0, thr, variant=v)
+                np.testing.assert_array_equal(host(har), want, err_msg=f"fused {mode} {v} thr={thr}")
+
+
 def test_harris_const_range(isp):
     d = dev(np.zeros((8, 16), dtype=np.int16))
     with pytest.raises(isp.IspError):
