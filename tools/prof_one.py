@@ -23,7 +23,7 @@ def main():
     ap.add_argument("--size", type=int, default=4096)
     ap.add_argument("--window", type=int, default=5)
     ap.add_argument("--launches", type=int, default=4)
-    ap.add_argument("--op", default="gauss", choices=["gauss", "sobel", "laplace", "harris", "bilateral", "fused3"])
+    ap.add_argument("--op", default="gauss", choices=["gauss", "gauss_u8", "sobel", "laplace", "harris", "bilateral", "fused3"])
     a = ap.parse_args()
     n = a.size
     if a.op != "gauss":
@@ -42,6 +42,9 @@ def main():
             elif a.op == "fused3":
                 lap, har = torch.empty_like(u8), torch.empty_like(u8)
                 isp.isp_pipeline_cfg3_u8(u8, a.mode, mag=o8, lap=lap, harris=har, variant=a.variant)
+            elif a.op == "gauss_u8":
+                b5 = np.array([1, 4, 6, 4, 1], dtype=np.int32)
+                isp.isp_filter_u8(u8, np.outer(b5, b5).astype(np.int32), 256, a.mode, out=o8, variant=a.variant)
             elif a.op == "harris":
                 isp.isp_harris_u8(dx, dy, a.mode, out=o8, variant=a.variant)
             else:
