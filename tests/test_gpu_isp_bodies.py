@@ -574,7 +574,7 @@ def test_laplace_harris_tile_kernels(isp, shape):
 
 # ---------------------------------------------------------------- warp-strip band Laplace
 @pytest.mark.parametrize("nw", [4, 2])
-@pytest.mark.parametrize("shape", [(8, 32), (9, 48), (70, 2064), (33, 4112), (260, 528), (101, 512), (4096 // 8, 4096),
+@pytest.mark.parametrize("shape", [(8, 32), (9, 48), (9, 264), (70, 2064), (33, 4112), (260, 528), (101, 512), (4096 // 8, 4096),
                                    (17, 784)])
 def test_laplace_band_kernel(isp, shape, nw, monkeypatch):
     """The warp-strip streaming Laplace (band_u8.cu) at 16 and 8 pixels per lane: strips of
@@ -592,14 +592,15 @@ def test_laplace_band_kernel(isp, shape, nw, monkeypatch):
         for c in ((0, 255) if mode == "constant" else (0,)):
             got = host(isp.isp_laplace5_u8(d, mode, c, variant="tma"))
             p = isp.isp_last_plan()
-            assert p["choice"] == CODE["tma"] and p["tile_w"] == 128 * nw, p
+            # widths not a multiple of the lane's 4 nw pixels are not band-eligible (fallback)
+            assert (p["choice"] == CODE["tma"] and p["tile_w"] == 128 * nw) == (w % (4 * nw) == 0), p
             np.testing.assert_array_equal(got, oracle.laplace5_u8(img, mode, c), err_msg=f"{mode} c={c}")
     # AUTO (Eq. 10 decides between the band kernel and the naive one): still exact
     np.testing.assert_array_equal(host(isp.isp_laplace5_u8(d, "mirror", 0)), oracle.laplace5_u8(img, "mirror", 0))
 
 
 @pytest.mark.parametrize("groups", [1, 2])
-@pytest.mark.parametrize("shape", [(8, 16), (9, 136), (70, 2064), (33, 4112), (101, 256), (4096 // 8, 4096), (17, 264)])
+@pytest.mark.parametrize("shape", [(8, 16), (9, 132), (9, 136), (70, 2064), (33, 4112), (101, 256), (4096 // 8, 4096), (17, 264)])
 def test_harris_band_kernel(isp, shape, groups, monkeypatch):
     """The warp-strip streaming Harris (band_u8.cu): strips of 128 columns (partial last
     strips down to one lane, one strip that is both L and R), bands down to 4 rows, all
@@ -620,7 +621,8 @@ def test_harris_band_kernel(isp, shape, groups, monkeypatch):
                 for thr in (0, -(10 ** 9), 10 ** 8, 10 ** 13):
                     got = host(isp.isp_harris_u8(ddx, ddy, mode, c, thr, variant="tma"))
                     p = isp.isp_last_plan()
-                    assert p["choice"] == CODE["tma"] and p["warp_w"] == 128 * groups and p["tile_h"] < 32, p
+                    band = p["choice"] == CODE["tma"] and p["warp_w"] == 128 * groups and p["tile_h"] < 32
+                    assert band == (w % (4 * groups) == 0), p   # partial lanes: not band-eligible
                     np.testing.assert_array_equal(got, oracle.harris(dx, dy, mode, c, thr),
                                                   err_msg=f"{mode} c={c} thr={thr}")
 
@@ -651,7 +653,7 @@ def test_sep_band_kernel(isp, shape, m):
 
 # ---------------------------------------------------------------- warp-strip band Sobel
 @pytest.mark.parametrize("groups", [1, 2])
-@pytest.mark.parametrize("shape", [(8, 16), (9, 136), (70, 2064), (45, 264), (4096 // 8, 4096)])
+@pytest.mark.parametrize("shape", [(8, 16), (9, 132), (9, 136), (70, 2064), (45, 264), (4096 // 8, 4096)])
 def test_sobel_band_kernel(isp, shape, groups, monkeypatch):
     """k_sob_band (band_u8.cu), the TMA / AUTO kernel of isp_sobel_u8: strips of 128
     columns (partial last strips down to one lane, one strip that is L and R), all modes and
@@ -669,7 +671,8 @@ def test_sobel_band_kernel(isp, shape, groups, monkeypatch):
             for want in (("dx", "dy", "mag"), ("mag",), ("dx",), ("dy", "mag")):
                 dx, dy, mag = isp.isp_sobel_u8(d, mode, c, variant="tma", want=want)
                 p = isp.isp_last_plan()
-                assert p["choice"] == CODE["tma"] and p["warp_w"] == 128 * groups and p["tile_h"] < 32, p
+                band = p["choice"] == CODE["tma"] and p["warp_w"] == 128 * groups and p["tile_h"] < 32
+                assert band == (w % (4 * groups) == 0), p   # partial lanes: not band-eligible
                 for name, got, ref in (("dx", dx, rdx), ("dy", dy, rdy), ("mag", mag, rmag)):
                     if name in want:
                         np.testing.assert_array_equal(host(got), ref, err_msg=f"{name} {mode} c={c} {want}")
@@ -677,7 +680,7 @@ def test_sobel_band_kernel(isp, shape, groups, monkeypatch):
 
 # ---------------------------------------------------------------- warp-strip band separable u8
 @pytest.mark.parametrize("nw", [2, 4])
-@pytest.mark.parametrize("shape", [(8, 32), (9, 48), (70, 2064), (33, 4112), (260, 528), (4096 // 8, 4096)])
+@pytest.mark.parametrize("shape", [(8, 32), (9, 48), (9, 264), (70, 2064), (33, 4112), (260, 528), (4096 // 8, 4096)])
 def test_sepu8_band_kernel(isp, shape, nw, monkeypatch):
     """k_sepu8_band (band_u8.cu), the TMA / AUTO kernel of normalised separable u8 masks: the
     3x3 / 16 and 5x5 / 256 binomials and a [1,2,1]^2 / 32 mask (result <= 127), all modes,
@@ -696,7 +699,8 @@ def test_sepu8_band_kernel(isp, shape, nw, monkeypatch):
             ref = oracle.filter_u8(img, mask, div, mode, 201)
             got = host(isp.isp_filter_u8(d, mask, div, mode, 201, variant="tma"))
             p = isp.isp_last_plan()
-            assert p["choice"] == CODE["tma"] and p["warp_w"] == 128 * nw and p["tile_h"] < 32, p
+            band = p["choice"] == CODE["tma"] and p["warp_w"] == 128 * nw and p["tile_h"] < 32
+            assert band == (w % (4 * nw) == 0), p   # partial lanes: not band-eligible
             np.testing.assert_array_equal(got, ref, err_msg=f"{mode} div={div} m={mask.shape}")
     mask, _ = oracle.gaussian_u8_mask(5)
     got = host(isp.isp_filter_u8(d, mask, 300, "mirror", 0, variant="tma"))
