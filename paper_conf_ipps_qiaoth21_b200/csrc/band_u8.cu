@@ -328,6 +328,30 @@ __device__ __forceinline__ void harris2p(float2 sxx, float2 syy, float2 sxy, flo
     }
 }
 
+// harris2p for the pairs E and O of four pixels with one warp vote (same decisions)
+__device__ __forceinline__ uint32_t harris4v(float2 sxxE, float2 syyE, float2 sxyE, float2 sxxO, float2 syyO,
+                                             float2 sxyO, float thr_f, float thr_err, double thr)
+{
+    const float2 c = f2(1.14552676677703857421875e-05f, 1.14552676677703857421875e-05f), te = f2(thr_err, thr_err);
+    const float2 ntf = f2(-thr_f, -thr_f), k25 = f2(25.f, 25.f);
+    const float2 tE = add2(sxxE, syyE), tO = add2(sxxO, syyO);
+    const float2 ttE = mul2(tE, tE), ttO = mul2(tO, tO);
+    const float2 RE = fma2(k25, fma2(f2(-sxyE.x, -sxyE.y), sxyE, mul2(sxxE, syyE)), f2(-ttE.x, -ttE.y));
+    const float2 RO = fma2(k25, fma2(f2(-sxyO.x, -sxyO.y), sxyO, mul2(sxxO, syyO)), f2(-ttO.x, -ttO.y));
+    const float2 bE = fma2(ttE, c, te), bO = fma2(ttO, c, te);
+    const float2 dE = add2(RE, ntf), dO = add2(RO, ntf);
+    uint32_t h0 = dE.x > 0.f ? 255u : 0u, h2 = dE.y > 0.f ? 255u : 0u;
+    uint32_t h1 = dO.x > 0.f ? 255u : 0u, h3 = dO.y > 0.f ? 255u : 0u;
+    const bool u0 = fabsf(dE.x) < bE.x, u2 = fabsf(dE.y) < bE.y, u1 = fabsf(dO.x) < bO.x, u3 = fabsf(dO.y) < bO.y;
+    if (__any_sync(0xffffffffu, u0 || u1 || u2 || u3)) {
+        if (u0) h0 = ttE.x == 0.f ? (0.0 > thr ? 255u : 0u) : (uint32_t)harris_exact(sxxE.x, syyE.x, sxyE.x, thr);
+        if (u2) h2 = ttE.y == 0.f ? (0.0 > thr ? 255u : 0u) : (uint32_t)harris_exact(sxxE.y, syyE.y, sxyE.y, thr);
+        if (u1) h1 = ttO.x == 0.f ? (0.0 > thr ? 255u : 0u) : (uint32_t)harris_exact(sxxO.x, syyO.x, sxyO.x, thr);
+        if (u3) h3 = ttO.y == 0.f ? (0.0 > thr ? 255u : 0u) : (uint32_t)harris_exact(sxxO.y, syyO.y, sxyO.y, thr);
+    }
+    return __byte_perm(__byte_perm(h0, h1, 0x0040), __byte_perm(h2, h3, 0x0040), 0x5410);
+}
+
 template <int G, bool CY>
 __device__ __forceinline__ void har_band_body(const HarBandParams &p, uint32_t ring, int xs0, int y0, int rows,
                                               int lane, bool cl, bool cr)
@@ -716,12 +740,8 @@ __device__ __forceinline__ void fused_band_body(const FusedBandParams &p, uint32
                         const float2 sxxE = add2(acc.xxE, hn.xxE), sxxO = add2(acc.xxO, hn.xxO);
                         const float2 syyE = add2(acc.yyE, hn.yyE), syyO = add2(acc.yyO, hn.yyO);
                         const float2 sxyE = add2(acc.xyE, hn.xyE), sxyO = add2(acc.xyO, hn.xyO);
-                        uint32_t h0, h1, h2, h3;
-                        harris2p(sxxE, syyE, sxyE, p.thr_f, p.thr_err, p.thr, h0, h2);
-                        harris2p(sxxO, syyO, sxyO, p.thr_f, p.thr_err, p.thr, h1, h3);
-                        if (active)
-                            *reinterpret_cast<uint32_t *>(p.har + o4) =
-                                __byte_perm(__byte_perm(h0, h1, 0x0040), __byte_perm(h2, h3, 0x0040), 0x5410);
+                        const uint32_t hw = harris4v(sxxE, syyE, sxyE, sxxO, syyO, sxyO, p.thr_f, p.thr_err, p.thr);
+                        if (active) *reinterpret_cast<uint32_t *>(p.har + o4) = hw;
                     }
                     // vertical [1,2,1] as a running pair (two rows of state instead of three;
                     // integer sums < 2^24, exact in any order)
