@@ -583,7 +583,7 @@ __device__ __forceinline__ uint32_t mag_bits(float n)
     return __float_as_uint(r + 8388608.0f);   // low byte = round(r) <= 255
 }
 
-template <bool CY>
+template <bool CY, bool DXY>
 __device__ __forceinline__ void fused_band_body(const FusedBandParams &p, uint32_t ring, int xs0, int y0, int rows,
                                                 int lane, bool cl, bool cr)
 {
@@ -723,7 +723,7 @@ __device__ __forceinline__ void fused_band_body(const FusedBandParams &p, uint32
                         const uint32_t m0 = mag_bits(nE.x), m1 = mag_bits(nO.x), m2 = mag_bits(nE.y), m3 = mag_bits(nO.y);
                         const uint32_t mw = __byte_perm(__byte_perm(m0, m1, 0x0040), __byte_perm(m2, m3, 0x0040), 0x5410);
                         if (active) *reinterpret_cast<uint32_t *>(p.mag + o3) = mw;
-                        if (p.dx && active) {   // int16 = low half of the bits of v + 1.5 * 2^23
+                        if (DXY && active) {   // int16 = low half of the bits of v + 1.5 * 2^23
                             const float2 a2 = add2(xE, f2(12582912.f, 12582912.f)), b2 = add2(xO, f2(12582912.f, 12582912.f));
                             const float2 c2_ = add2(yE, f2(12582912.f, 12582912.f)), d2 = add2(yO, f2(12582912.f, 12582912.f));
                             *reinterpret_cast<uint2 *>(p.dx + o3) =
@@ -761,6 +761,7 @@ __device__ __forceinline__ void fused_band_body(const FusedBandParams &p, uint32
     }
 }
 
+template <bool DXY>
 __global__ void __launch_bounds__(NTB, FUSED_MINB) k_fused_band(const __grid_constant__ FusedBandParams p)
 {
     __shared__ __align__(16) uint8_t rings[BW][FLR * FSLOT];
@@ -775,8 +776,8 @@ __global__ void __launch_bounds__(NTB, FUSED_MINB) k_fused_band(const __grid_con
     band_rows(band, g.nband, g.h, y0, y1);
     const bool cl = s < g.sx0, cr = s >= g.sx1, cy = band < g.by0 || band >= g.by1;
     const uint32_t ring = su32(rings[warp]);
-    if (cy) fused_band_body<true>(p, ring, s * FSTRIP, y0, y1 - y0, lane, cl, cr);
-    else fused_band_body<false>(p, ring, s * FSTRIP, y0, y1 - y0, lane, cl, cr);
+    if (cy) fused_band_body<true, DXY>(p, ring, s * FSTRIP, y0, y1 - y0, lane, cl, cr);
+    else fused_band_body<false, DXY>(p, ring, s * FSTRIP, y0, y1 - y0, lane, cl, cr);
 }
 
 
@@ -1156,7 +1157,7 @@ int band_blocks_per_sm(int which)
     static int nb[5] = {-1, -1, -1, -1, -1};
     if (nb[which] < 0) {
         const void *fn = which == 1   ? har_band_fn(harris_g())
-                         : which == 3 ? (const void *)k_fused_band
+                         : which == 3 ? (const void *)k_fused_band<false>
                          : which == 0 ? sob_band_fn(sobel_g())
                                       : lap_band_fn(which);
         if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb[which], fn, NTB, 0) != cudaSuccess) {
@@ -1267,7 +1268,8 @@ cudaError_t ispi_fused_band(const uint8_t *img, int w, int h, int pitch, int mod
     p.thr = (double)std::max(-9007199254740992ll, std::min(9007199254740992ll, thr));
     p.thr_f = (float)p.thr;
     p.thr_err = thr_bound(p.thr_f);
-    return launch_band((const void *)k_fused_band, &p, p.g.ngx * p.g.nband, st);
+    return launch_band(p.dx ? (const void *)k_fused_band<true> : (const void *)k_fused_band<false>, &p,
+                       p.g.ngx * p.g.nband, st);
 }
 
 // Sobel band kernel: 4 G-pixel lane granules, 4 G-byte aligned input and mag rows, 8 G-byte
