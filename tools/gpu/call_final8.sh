@@ -1,4 +1,4 @@
-# Final measurement after the fused kernel's single Harris vote: GPU suite, traffic of the
+# Final measurement (fused: single Harris vote, dx / dy outputs as a template parameter): GPU suite, traffic of the
 # in-tree library, bench lines, fused / u8 timings, the fused ncu capture
 set -x
 md5sum paper_conf_ipps_qiaoth21_b200/libisp.so
